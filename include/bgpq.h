@@ -1,0 +1,126 @@
+/* include/bgpq.h — C ABI of the B200-native BGPQ batched-heap priority queue.
+ *
+ * The operations are those of the paper's problem statement (BGPQ, Chen et al., ICPP'21,
+ * /root/reference/PAPER.md, cited as P:<line>):
+ *   - the priority-queue ADT: INSERT of (key, value) pairs and DELETEMIN returning the pair
+ *     with the smallest key (§2);
+ *   - batched: one INSERT carries 1..k keys, one DELETEMIN returns the 1..k smallest keys,
+ *     or every key left if fewer remain (§3.2);
+ *   - linearizable: every operation takes effect at a point while it holds the root lock
+ *     (§5).
+ *
+ * Conventions common to every call
+ *   - Keys and values are uint32; keys are ordered as unsigned integers ("32-bit keys").
+ *   - All key / value / count pointers are DEVICE pointers unless the name ends in _host.
+ *   - `stream` is a cudaStream_t passed as void* (NULL = legacy default stream).  Calls are
+ *     asynchronous and stream-ordered; caller buffers must stay valid until the stream has
+ *     reached the call (as with cudaMemcpyAsync).  One handle must not be used from two
+ *     streams concurrently: concurrency lives INSIDE a call (many CTAs execute its batch
+ *     operations at once) and in bgpq_run_mixed.
+ *   - The handle owns the heap storage; the caller owns every other buffer.
+ *   - Return values: BGPQ_OK (0) or a negative BGPQ_E* code.  bgpq_create returns NULL on
+ *     failure; bgpq_last_error() then says why (thread-local).
+ *   - There is no CPU fallback: if no sm_100 device is present the calls fail with
+ *     BGPQ_ECUDA.
+ */
+#ifndef BGPQ_H
+#define BGPQ_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct bgpq bgpq_t;
+
+enum {
+  BGPQ_OK = 0,
+  BGPQ_EINVAL = -1, /* bad argument (K not in {64,128,256,512,1024}, NULL pointer, ...) */
+  BGPQ_ENOMEM = -2, /* device allocation failed                                          */
+  BGPQ_EFULL = -3,  /* sticky: an INSERT needed a node beyond the capacity; op dropped   */
+  BGPQ_ECUDA = -4   /* a CUDA runtime call or kernel launch failed                       */
+};
+
+/* bgpq_create_ex flags */
+enum {
+  BGPQ_FLAG_VALUES = 1u, /* store a uint32 value with every key (w = 8 B per entry)        */
+  BGPQ_FLAG_SERIAL = 2u  /* execute operations one at a time on a single CTA (test mode:
+                            the node layout then equals the sequential Alg.1-3 model)     */
+};
+
+/* Create an empty heap able to hold `capacity` keys with node capacity K (§3.1:
+ * every non-root node holds K sorted keys; k > 1).  K must be one of 64, 128, 256, 512,
+ * 1024.  Allocates ceil(capacity/K)+2 node slots of K entries in device memory of the
+ * current device.  bgpq_create stores keys and values (flags = BGPQ_FLAG_VALUES). */
+bgpq_t* bgpq_create(uint64_t capacity, uint32_t K);
+bgpq_t* bgpq_create_ex(uint64_t capacity, uint32_t K, uint32_t flags);
+
+/* Free the handle and its device memory (synchronizes the device first). */
+void bgpq_destroy(bgpq_t* q);
+
+/* INSERT n keys (Alg.1 BGPQ_INSERT): executed as ceil(n/K) batch INSERTs of
+ * the consecutive K-slices keys[j*K, min(n,(j+1)*K)), linearized in some order.
+ * keys: device, n entries.  vals: device, n entries, or NULL (values then undefined; a
+ * handle without BGPQ_FLAG_VALUES ignores vals).  n = 0 is a no-op.
+ * Capacity overflow sets the sticky BGPQ_EFULL reported by bgpq_size(); the overflowing
+ * batch is dropped. */
+int bgpq_insert(bgpq_t* q, const uint32_t* keys, const uint32_t* vals, uint64_t n, void* stream);
+
+/* DELETEMIN n keys (Alg.2+3): executed as ceil(n/K) batch DELETEMINs.  The
+ * batch that takes linearization ticket t of this call asks for min(K, n - t*K) keys and
+ * writes them at out_keys[t*K ...], so the output is compact and ascending when no INSERT
+ * runs concurrently.  Writes min(n, current size) entries in total; if d_count != NULL
+ * (device uint64) that count is ADDED to *d_count.  out_vals may be NULL. */
+int bgpq_deletemin(bgpq_t* q, uint32_t* out_keys, uint32_t* out_vals, uint64_t n,
+                   uint64_t* d_count, void* stream);
+
+/* Number of keys in the heap (|root| + |pBuffer| + K*(heapSize-1)).  Synchronizes
+ * `stream`.  Returns BGPQ_EFULL if a capacity overflow happened since creation. */
+int bgpq_size(bgpq_t* q, uint64_t* out_size, void* stream);
+
+/* Same as bgpq_insert / bgpq_deletemin with HOST buffers (pinned memory gives full
+ * PCIe bandwidth): the host->device and device->host copies are part of the call and are
+ * ordered on `stream`; the call returns after the results are in the host buffers.
+ * out_count_host (nullable) receives the number of entries written. */
+int bgpq_insert_host(bgpq_t* q, const uint32_t* keys_host, const uint32_t* vals_host, uint64_t n,
+                     void* stream);
+int bgpq_deletemin_host(bgpq_t* q, uint32_t* out_keys_host, uint32_t* out_vals_host, uint64_t n,
+                        uint64_t* out_count_host, void* stream);
+
+/* Test / bench extension: run an arbitrary stream of n_ops batch operations concurrently
+ * on the persistent CTAs (op j: op_types[j] 0 = INSERT, 1 = DELETEMIN; op_sizes[j] in 1..K).
+ * INSERT j reads op_sizes[j] keys at in_keys[in_off[j]]; DELETEMIN j writes at
+ * out_keys[j*K] and its entry count to op_count[j].  lin_ticket[j] (nullable) receives
+ * the global linearization ticket taken under the root lock.  All device. */
+int bgpq_run_mixed(bgpq_t* q, const uint8_t* op_types, const uint32_t* op_sizes,
+                   const uint64_t* in_off, uint64_t n_ops, const uint32_t* in_keys,
+                   const uint32_t* in_vals, uint32_t* out_keys, uint32_t* out_vals,
+                   uint32_t* op_count, uint64_t* lin_ticket, void* stream);
+
+/* Test extension: copy the quiescent heap to HOST buffers.  node_keys / node_vals:
+ * (slots)*K entries, slot 0 = pBuffer, slot 1 = root, slot i >= 2 = node i; meta: 4
+ * uint32 per slot {lock, state (0 EMPTY, 1 AVAIL, 2 TARGET, 3 MARKED), min, max};
+ * hdr: {heapSize, |root|, |pBuffer|, sticky error}.  Synchronizes the device. */
+int bgpq_dump(bgpq_t* q, uint32_t* node_keys, uint32_t* node_vals, uint32_t* meta, uint64_t* hdr);
+uint64_t bgpq_slots(bgpq_t* q); /* number of node slots (= max node index + 1) */
+
+/* Device counters accumulated over the handle's lifetime (for the byte model), written to
+ * out[0..n): see BGPQ_STAT_* in DESIGN.md.  Synchronizes the device. */
+int bgpq_stats(bgpq_t* q, uint64_t* out, int n);
+
+/* Grid control: ctas = 0 -> all co-resident CTAs (default), 1 -> serialized. */
+int bgpq_set_grid(bgpq_t* q, int ctas);
+int bgpq_grid(bgpq_t* q);
+
+/* Number of kernels this library has launched in the process (for bench gpu_launches). */
+uint64_t bgpq_launch_count(void);
+
+int bgpq_last_error(void);
+const char* bgpq_strerror(int code);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* BGPQ_H */

@@ -1,0 +1,370 @@
+// bgpq_api.cu — host side of the C ABI declared in include/bgpq.h.
+// Owns the heap arena (node keys/values, node metadata, header), validates arguments,
+// dispatches on the node capacity K (template instantiations 64..1024, keys-only or
+// key+value) and launches the persistent ops kernel on the caller's stream.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <atomic>
+#include <cstdio>
+#include <cstring>
+
+#include "../../include/bgpq.h"
+#include "bgpq_ops.cuh"
+
+using namespace bgpqd;
+
+namespace {
+
+constexpr int NT = 512;  // threads per CTA (the paper's block size)
+
+thread_local int g_last_error = BGPQ_OK;
+std::atomic<unsigned long long> g_launches{0};
+
+int fail(int code) {
+  g_last_error = code;
+  return code;
+}
+
+}  // namespace
+
+struct bgpq {
+  int device = 0;
+  u32 K = 0;
+  u32 flags = 0;
+  u64 capacity = 0;
+  u32 cap_nodes = 0;  // largest node index
+  u64 slots = 0;      // cap_nodes + 1
+  u32* gk = nullptr;
+  u32* gv = nullptr;
+  NodeMeta* meta = nullptr;
+  u32* hdr = nullptr;
+  int sm_count = 0;
+  int occ = 0;         // co-resident CTAs per SM for this K
+  int grid_req = 0;    // 0 auto, else exact
+  u32* stage_k = nullptr;  // staging for the *_host calls
+  u32* stage_v = nullptr;
+  u64* stage_cnt = nullptr;
+  u64 stage_n = 0;
+};
+
+namespace {
+
+template <int K, bool V>
+struct KernelInfo {
+  static int occupancy(int* out_occ) {
+    auto kern = bgpq_ops_kernel<K, V, NT>;
+    const size_t smem = ops_smem_bytes<K, V>();
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return -1;
+    int occ = 0;
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, NT, smem);
+    if (e != cudaSuccess) return -1;
+    *out_occ = occ;
+    return 0;
+  }
+  static cudaError_t launch(int grid, const HeapArgs& H, const CallArgs& C, cudaStream_t s) {
+    bgpq_ops_kernel<K, V, NT><<<grid, NT, ops_smem_bytes<K, V>(), s>>>(H, C);
+    g_launches.fetch_add(1);
+    return cudaGetLastError();
+  }
+};
+
+int occupancy_for(u32 K, bool V, int* occ) {
+#define BGPQ_CASE(KK)                                                                \
+  case KK:                                                                           \
+    return V ? KernelInfo<KK, true>::occupancy(occ) : KernelInfo<KK, false>::occupancy(occ);
+  switch (K) {
+    BGPQ_CASE(64)
+    BGPQ_CASE(128)
+    BGPQ_CASE(256)
+    BGPQ_CASE(512)
+    BGPQ_CASE(1024)
+    default:
+      return -1;
+  }
+#undef BGPQ_CASE
+}
+
+cudaError_t launch_for(u32 K, bool V, int grid, const HeapArgs& H, const CallArgs& C, cudaStream_t s) {
+#define BGPQ_CASE(KK)                                                                        \
+  case KK:                                                                                   \
+    return V ? KernelInfo<KK, true>::launch(grid, H, C, s) : KernelInfo<KK, false>::launch(grid, H, C, s);
+  switch (K) {
+    BGPQ_CASE(64)
+    BGPQ_CASE(128)
+    BGPQ_CASE(256)
+    BGPQ_CASE(512)
+    BGPQ_CASE(1024)
+    default:
+      return cudaErrorInvalidValue;
+  }
+#undef BGPQ_CASE
+}
+
+bool valid_K(u32 K) { return K == 64 || K == 128 || K == 256 || K == 512 || K == 1024; }
+
+HeapArgs heap_args(const bgpq* q) {
+  HeapArgs H;
+  H.gk = q->gk;
+  H.gv = (q->flags & BGPQ_FLAG_VALUES) ? q->gv : nullptr;
+  H.meta = q->meta;
+  H.hdr = q->hdr;
+  H.cap = q->cap_nodes;
+  return H;
+}
+
+int grid_for(const bgpq* q, u64 n_ops) {
+  if (q->flags & BGPQ_FLAG_SERIAL) return 1;
+  long long g = q->grid_req > 0 ? q->grid_req : (long long)q->sm_count * q->occ;
+  if ((u64)g > n_ops) g = (long long)n_ops;
+  return (int)std::max(1LL, g);
+}
+
+int run_call(bgpq* q, const CallArgs& C, cudaStream_t s) {
+  // reset the per-call ticket and fetch counter (header words H_CALL, H_FETCH)
+  if (cudaMemsetAsync(q->hdr + H_CALL, 0, 2 * sizeof(u32), s) != cudaSuccess) return fail(BGPQ_ECUDA);
+  const bool V = (q->flags & BGPQ_FLAG_VALUES) != 0;
+  if (launch_for(q->K, V, grid_for(q, C.n_ops), heap_args(q), C, s) != cudaSuccess) return fail(BGPQ_ECUDA);
+  return BGPQ_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+bgpq_t* bgpq_create_ex(uint64_t capacity, uint32_t K, uint32_t flags) {
+  g_last_error = BGPQ_OK;
+  if (!valid_K(K) || capacity == 0 || (flags & ~3u)) {
+    fail(BGPQ_EINVAL);
+    return nullptr;
+  }
+  bgpq* q = new bgpq();
+  q->K = K;
+  q->flags = flags;
+  q->capacity = capacity;
+  const u64 nodes = (capacity + K - 1) / K + 1;
+  if (nodes + 1 > 0xFFFFFFF0ull) {
+    delete q;
+    fail(BGPQ_EINVAL);
+    return nullptr;
+  }
+  q->cap_nodes = (u32)std::max<u64>(2, nodes);
+  q->slots = (u64)q->cap_nodes + 1;
+  if (cudaGetDevice(&q->device) != cudaSuccess ||
+      cudaDeviceGetAttribute(&q->sm_count, cudaDevAttrMultiProcessorCount, q->device) != cudaSuccess) {
+    delete q;
+    fail(BGPQ_ECUDA);
+    return nullptr;
+  }
+  const bool V = (flags & BGPQ_FLAG_VALUES) != 0;
+  if (occupancy_for(K, V, &q->occ) != 0 || q->occ < 1) {
+    delete q;
+    fail(BGPQ_ECUDA);
+    return nullptr;
+  }
+  const size_t nbytes = q->slots * (size_t)K * sizeof(u32);
+  bool ok = cudaMalloc(&q->gk, nbytes) == cudaSuccess;
+  if (ok && V) ok = cudaMalloc(&q->gv, nbytes) == cudaSuccess;
+  if (ok) ok = cudaMalloc(&q->meta, q->slots * sizeof(NodeMeta)) == cudaSuccess;
+  if (ok) ok = cudaMalloc(&q->hdr, HEADER_WORDS * sizeof(u32)) == cudaSuccess;
+  if (ok) ok = cudaMemset(q->meta, 0, q->slots * sizeof(NodeMeta)) == cudaSuccess;
+  if (ok) ok = cudaMemset(q->hdr, 0, HEADER_WORDS * sizeof(u32)) == cudaSuccess;
+  if (ok) ok = cudaDeviceSynchronize() == cudaSuccess;
+  if (!ok) {
+    cudaGetLastError();
+    bgpq_destroy(q);
+    fail(BGPQ_ENOMEM);
+    return nullptr;
+  }
+  return q;
+}
+
+bgpq_t* bgpq_create(uint64_t capacity, uint32_t K) { return bgpq_create_ex(capacity, K, BGPQ_FLAG_VALUES); }
+
+void bgpq_destroy(bgpq_t* q) {
+  if (!q) return;
+  cudaDeviceSynchronize();
+  cudaFree(q->gk);
+  cudaFree(q->gv);
+  cudaFree(q->meta);
+  cudaFree(q->hdr);
+  cudaFree(q->stage_k);
+  cudaFree(q->stage_v);
+  cudaFree(q->stage_cnt);
+  delete q;
+}
+
+int bgpq_insert(bgpq_t* q, const uint32_t* keys, const uint32_t* vals, uint64_t n, void* stream) {
+  if (!q) return fail(BGPQ_EINVAL);
+  if (n == 0) return BGPQ_OK;
+  if (!keys) return fail(BGPQ_EINVAL);
+  CallArgs C;
+  memset(&C, 0, sizeof(C));
+  C.mode = MODE_INSERT;
+  C.n = n;
+  C.n_ops = (n + q->K - 1) / q->K;
+  C.in_k = keys;
+  C.in_v = (q->flags & BGPQ_FLAG_VALUES) ? vals : nullptr;
+  return run_call(q, C, (cudaStream_t)stream);
+}
+
+int bgpq_deletemin(bgpq_t* q, uint32_t* out_keys, uint32_t* out_vals, uint64_t n, uint64_t* d_count,
+                   void* stream) {
+  if (!q) return fail(BGPQ_EINVAL);
+  if (n == 0) return BGPQ_OK;
+  if (!out_keys) return fail(BGPQ_EINVAL);
+  CallArgs C;
+  memset(&C, 0, sizeof(C));
+  C.mode = MODE_DELETEMIN;
+  C.n = n;
+  C.n_ops = (n + q->K - 1) / q->K;
+  C.out_k = out_keys;
+  C.out_v = (q->flags & BGPQ_FLAG_VALUES) ? out_vals : nullptr;
+  C.d_count = reinterpret_cast<ull*>(d_count);
+  return run_call(q, C, (cudaStream_t)stream);
+}
+
+int bgpq_run_mixed(bgpq_t* q, const uint8_t* op_types, const uint32_t* op_sizes, const uint64_t* in_off,
+                   uint64_t n_ops, const uint32_t* in_keys, const uint32_t* in_vals, uint32_t* out_keys,
+                   uint32_t* out_vals, uint32_t* op_count, uint64_t* lin_ticket, void* stream) {
+  if (!q) return fail(BGPQ_EINVAL);
+  if (n_ops == 0) return BGPQ_OK;
+  if (!op_types || !op_sizes || !in_off || !in_keys || !out_keys || !op_count) return fail(BGPQ_EINVAL);
+  CallArgs C;
+  memset(&C, 0, sizeof(C));
+  C.mode = MODE_MIXED;
+  C.n_ops = n_ops;
+  C.op_types = op_types;
+  C.op_sizes = op_sizes;
+  C.in_off = reinterpret_cast<const u64*>(in_off);
+  C.in_k = in_keys;
+  C.in_v = (q->flags & BGPQ_FLAG_VALUES) ? in_vals : nullptr;
+  C.out_k = out_keys;
+  C.out_v = (q->flags & BGPQ_FLAG_VALUES) ? out_vals : nullptr;
+  C.op_count = op_count;
+  C.lin_ticket = reinterpret_cast<ull*>(lin_ticket);
+  return run_call(q, C, (cudaStream_t)stream);
+}
+
+int bgpq_size(bgpq_t* q, uint64_t* out_size, void* stream) {
+  if (!q || !out_size) return fail(BGPQ_EINVAL);
+  u32 h[4];
+  cudaStream_t s = (cudaStream_t)stream;
+  if (cudaMemcpyAsync(h, q->hdr, sizeof(h), cudaMemcpyDeviceToHost, s) != cudaSuccess ||
+      cudaStreamSynchronize(s) != cudaSuccess)
+    return fail(BGPQ_ECUDA);
+  *out_size = h[H_HS] == 0 ? 0 : (u64)h[H_RS] + h[H_PS] + (u64)(h[H_HS] - 1) * q->K;
+  if (h[H_ERR]) return fail((int)h[H_ERR]);
+  return BGPQ_OK;
+}
+
+static int ensure_stage(bgpq* q, u64 n) {
+  if (q->stage_n >= n) return BGPQ_OK;
+  cudaFree(q->stage_k);
+  cudaFree(q->stage_v);
+  q->stage_k = q->stage_v = nullptr;
+  if (!q->stage_cnt && cudaMalloc(&q->stage_cnt, sizeof(u64)) != cudaSuccess) return fail(BGPQ_ENOMEM);
+  if (cudaMalloc(&q->stage_k, n * sizeof(u32)) != cudaSuccess) return fail(BGPQ_ENOMEM);
+  if ((q->flags & BGPQ_FLAG_VALUES) && cudaMalloc(&q->stage_v, n * sizeof(u32)) != cudaSuccess)
+    return fail(BGPQ_ENOMEM);
+  q->stage_n = n;
+  return BGPQ_OK;
+}
+
+int bgpq_insert_host(bgpq_t* q, const uint32_t* keys_host, const uint32_t* vals_host, uint64_t n, void* stream) {
+  if (!q || (n && !keys_host)) return fail(BGPQ_EINVAL);
+  if (n == 0) return BGPQ_OK;
+  int rc = ensure_stage(q, n);
+  if (rc) return rc;
+  cudaStream_t s = (cudaStream_t)stream;
+  const bool V = (q->flags & BGPQ_FLAG_VALUES) && vals_host;
+  if (cudaMemcpyAsync(q->stage_k, keys_host, n * 4, cudaMemcpyHostToDevice, s) != cudaSuccess) return fail(BGPQ_ECUDA);
+  if (V && cudaMemcpyAsync(q->stage_v, vals_host, n * 4, cudaMemcpyHostToDevice, s) != cudaSuccess)
+    return fail(BGPQ_ECUDA);
+  rc = bgpq_insert(q, q->stage_k, V ? q->stage_v : nullptr, n, stream);
+  if (rc) return rc;
+  if (cudaStreamSynchronize(s) != cudaSuccess) return fail(BGPQ_ECUDA);
+  return BGPQ_OK;
+}
+
+int bgpq_deletemin_host(bgpq_t* q, uint32_t* out_keys_host, uint32_t* out_vals_host, uint64_t n,
+                        uint64_t* out_count_host, void* stream) {
+  if (!q || (n && !out_keys_host)) return fail(BGPQ_EINVAL);
+  if (n == 0) {
+    if (out_count_host) *out_count_host = 0;
+    return BGPQ_OK;
+  }
+  int rc = ensure_stage(q, n);
+  if (rc) return rc;
+  cudaStream_t s = (cudaStream_t)stream;
+  const bool V = (q->flags & BGPQ_FLAG_VALUES) && out_vals_host;
+  if (cudaMemsetAsync(q->stage_cnt, 0, sizeof(u64), s) != cudaSuccess) return fail(BGPQ_ECUDA);
+  rc = bgpq_deletemin(q, q->stage_k, V ? q->stage_v : nullptr, n, q->stage_cnt, stream);
+  if (rc) return rc;
+  u64 cnt = 0;
+  if (cudaMemcpyAsync(&cnt, q->stage_cnt, sizeof(u64), cudaMemcpyDeviceToHost, s) != cudaSuccess ||
+      cudaStreamSynchronize(s) != cudaSuccess)
+    return fail(BGPQ_ECUDA);
+  if (cnt && cudaMemcpyAsync(out_keys_host, q->stage_k, cnt * 4, cudaMemcpyDeviceToHost, s) != cudaSuccess)
+    return fail(BGPQ_ECUDA);
+  if (cnt && V && cudaMemcpyAsync(out_vals_host, q->stage_v, cnt * 4, cudaMemcpyDeviceToHost, s) != cudaSuccess)
+    return fail(BGPQ_ECUDA);
+  if (cudaStreamSynchronize(s) != cudaSuccess) return fail(BGPQ_ECUDA);
+  if (out_count_host) *out_count_host = cnt;
+  return BGPQ_OK;
+}
+
+uint64_t bgpq_slots(bgpq_t* q) { return q ? q->slots : 0; }
+
+int bgpq_dump(bgpq_t* q, uint32_t* node_keys, uint32_t* node_vals, uint32_t* meta, uint64_t* hdr) {
+  if (!q) return fail(BGPQ_EINVAL);
+  if (cudaDeviceSynchronize() != cudaSuccess) return fail(BGPQ_ECUDA);
+  const size_t nbytes = q->slots * (size_t)q->K * sizeof(u32);
+  if (node_keys && cudaMemcpy(node_keys, q->gk, nbytes, cudaMemcpyDeviceToHost) != cudaSuccess) return fail(BGPQ_ECUDA);
+  if (node_vals && q->gv && cudaMemcpy(node_vals, q->gv, nbytes, cudaMemcpyDeviceToHost) != cudaSuccess)
+    return fail(BGPQ_ECUDA);
+  if (meta && cudaMemcpy(meta, q->meta, q->slots * sizeof(NodeMeta), cudaMemcpyDeviceToHost) != cudaSuccess)
+    return fail(BGPQ_ECUDA);
+  if (hdr) {
+    u32 h[4];
+    if (cudaMemcpy(h, q->hdr, sizeof(h), cudaMemcpyDeviceToHost) != cudaSuccess) return fail(BGPQ_ECUDA);
+    for (int i = 0; i < 4; ++i) hdr[i] = h[i];
+  }
+  return BGPQ_OK;
+}
+
+int bgpq_stats(bgpq_t* q, uint64_t* out, int n) {
+  if (!q || !out || n < 0) return fail(BGPQ_EINVAL);
+  if (cudaDeviceSynchronize() != cudaSuccess) return fail(BGPQ_ECUDA);
+  ull st[NSTAT];
+  if (cudaMemcpy(st, q->hdr + H_STAT, sizeof(st), cudaMemcpyDeviceToHost) != cudaSuccess) return fail(BGPQ_ECUDA);
+  for (int i = 0; i < n && i < NSTAT; ++i) out[i] = st[i];
+  return BGPQ_OK;
+}
+
+int bgpq_set_grid(bgpq_t* q, int ctas) {
+  if (!q || ctas < 0) return fail(BGPQ_EINVAL);
+  if (ctas > q->sm_count * q->occ) return fail(BGPQ_EINVAL);  // must stay co-resident
+  q->grid_req = ctas;
+  return BGPQ_OK;
+}
+
+int bgpq_grid(bgpq_t* q) { return q ? grid_for(q, ~0ull) : 0; }
+
+uint64_t bgpq_launch_count(void) { return g_launches.load(); }
+
+int bgpq_last_error(void) { return g_last_error; }
+
+const char* bgpq_strerror(int code) {
+  switch (code) {
+    case BGPQ_OK: return "ok";
+    case BGPQ_EINVAL: return "invalid argument";
+    case BGPQ_ENOMEM: return "device allocation failed";
+    case BGPQ_EFULL: return "capacity exceeded (sticky; the overflowing batch was dropped)";
+    case BGPQ_ECUDA: return "CUDA error";
+    default: return "unknown error";
+  }
+}
+
+}  // extern "C"

@@ -1,0 +1,238 @@
+// bgpq_prim.cuh — sm_100a device primitives for the BGPQ hot path.
+//
+//  * PTX wrappers: acquire/release node locks (atom.cas.acquire.gpu / st.release.gpu),
+//    relaxed/acquire loads, mbarrier + cp.async.bulk (TMA bulk) global->shared staging,
+//    proxy fences.
+//  * warp_sort64: in-register bitonic sort of 64-entry runs with __shfl_xor_sync
+//    ("Sort(items)", Alg.1 l.2 = P:203; bitonic sort [22]).
+//  * cta_merge_split: merge-path [11] partitioned merge of two sorted smem tiles,
+//    split at Ma — the SORT_SPLIT of P:196-198.
+//  * cta_sort: warp_sort64 runs followed by merge-path passes in smem.
+#pragma once
+#include <cstdint>
+
+namespace bgpqd {
+
+typedef uint32_t u32;
+typedef uint64_t u64;
+typedef unsigned long long ull;
+
+constexpr u32 KEY_MAX = 0xFFFFFFFFu;
+
+// ----------------------------------------------------------------------------------------
+// PTX wrappers
+// ----------------------------------------------------------------------------------------
+__device__ __forceinline__ u32 smem_addr(const void* p) {
+  return static_cast<u32>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ u32 ld_relaxed(const u32* p) {
+  u32 v;
+  asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ u32 ld_acquire(const u32* p) {
+  u32 v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_relaxed(u32* p, u32 v) {
+  asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ void st_release(u32* p, u32 v) {
+  asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ u32 cas_acquire(u32* p, u32 cmp, u32 val) {
+  u32 old;
+  asm volatile("atom.acquire.gpu.global.cas.b32 %0, [%1], %2, %3;"
+               : "=r"(old) : "l"(p), "r"(cmp), "r"(val) : "memory");
+  return old;
+}
+// generic <-> async proxy ordering (global and shared) — required between an acquire of a
+// node lock and the cp.async.bulk that reads the node, and before re-filling a smem tile
+// that generic-proxy code has touched.
+__device__ __forceinline__ void fence_proxy_async() {
+  asm volatile("fence.proxy.async;" ::: "memory");
+}
+
+// Node lock (D4): test-and-test-and-set with an acquire CAS; one elected thread spins
+// with __nanosleep backoff so the CAS traffic does not starve the holder's accesses.
+__device__ __forceinline__ u32 lock_acquire(u32* lk) {
+  u32 spins = 0, ns = 32;
+  for (;;) {
+    if (ld_relaxed(lk) == 0u && cas_acquire(lk, 0u, 1u) == 0u) return spins;
+    ++spins;
+    __nanosleep(ns);
+    ns = ns < 256 ? ns * 2 : 256;
+  }
+}
+// Release: the caller has made all of the CTA's writes to the protected data happen-before
+// this thread (by __syncthreads); the gpu-scope fence + release store publishes them.
+__device__ __forceinline__ void lock_release(u32* lk) {
+  __threadfence();
+  st_release(lk, 0u);
+}
+
+// mbarrier + TMA bulk copy (global -> shared), completion by transaction bytes.
+__device__ __forceinline__ void mbar_init(u64* bar, u32 count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_addr(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(u64* bar, u32 bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_addr(bar)),
+               "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(u64* bar, u32 phase) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n"
+      "WAIT_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+      "@!p bra WAIT_%=;\n}" ::"r"(smem_addr(bar)),
+      "r"(phase) : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, u32 bytes, u64* bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_addr(dst)),
+      "l"(src), "r"(bytes), "r"(smem_addr(bar)) : "memory");
+}
+
+// ----------------------------------------------------------------------------------------
+// Sort(items) — Alg.1 l.2, bitonic sort [22].
+// warp_sort64: one warp sorts 64 entries held two per lane (index e = lane + 32*s).
+// Comparison key = (key << 1) | is_pad so padding entries sort after real entries with
+// the same key; compare-exchange partners at distance j < 32 are fetched with
+// __shfl_xor_sync, the j = 32 partner is the lane's other register.
+// ----------------------------------------------------------------------------------------
+template <bool V>
+__device__ __forceinline__ void warp_sort64(u64& c0, u64& c1, u32& v0, u32& v1) {
+  const int lane = threadIdx.x & 31;
+#pragma unroll
+  for (int k = 2; k <= 64; k <<= 1) {
+#pragma unroll
+    for (int j = k >> 1; j > 0; j >>= 1) {
+      if (j == 32) {
+        // e0 = lane < 32 <= e1 = lane + 32, ascending iff ((e & k) == 0); k == 64 here
+        const bool asc = true;
+        const bool sw = asc ? (c1 < c0) : (c0 < c1);
+        if (sw) {
+          u64 t = c0; c0 = c1; c1 = t;
+          if (V) { u32 tv = v0; v0 = v1; v1 = tv; }
+        }
+      } else {
+        const u64 p0 = __shfl_xor_sync(0xffffffffu, c0, j);
+        const u64 p1 = __shfl_xor_sync(0xffffffffu, c1, j);
+        u32 q0 = 0, q1 = 0;
+        if (V) {
+          q0 = __shfl_xor_sync(0xffffffffu, v0, j);
+          q1 = __shfl_xor_sync(0xffffffffu, v1, j);
+        }
+        const int e0 = lane, e1 = lane + 32;
+        const bool lower = (lane & j) == 0;
+        const bool min0 = (lower == ((e0 & k) == 0));
+        const bool min1 = (lower == ((e1 & k) == 0));
+        const bool t0 = min0 ? (p0 < c0) : (p0 > c0);
+        const bool t1 = min1 ? (p1 < c1) : (p1 > c1);
+        if (t0) { c0 = p0; if (V) v0 = q0; }
+        if (t1) { c1 = p1; if (V) v1 = q1; }
+      }
+    }
+  }
+}
+
+// ----------------------------------------------------------------------------------------
+// SORT_SPLIT by merge path [11].
+// Z[0:na] and W[0:nb] are sorted smem tiles; the merged sequence (stable, Z before W on
+// equal keys) is written with its first `ma` entries to X and the rest to Y.
+// Each of the NT threads takes a contiguous range of output diagonals, finds its co-rank
+// by binary search on the diagonal and merges sequentially.  X/Y must not alias Z/W.
+// The caller synchronizes before and after.
+// ----------------------------------------------------------------------------------------
+template <int NT, bool V>
+__device__ __forceinline__ void cta_merge_split(const u32* __restrict__ zk, const u32* __restrict__ zv,
+                                                int na, const u32* __restrict__ wk,
+                                                const u32* __restrict__ wv, int nb, int ma,
+                                                u32* __restrict__ xk, u32* __restrict__ xv,
+                                                u32* __restrict__ yk, u32* __restrict__ yv) {
+  const int N = na + nb;
+  const int per = (N + NT - 1) / NT;
+  const int d = threadIdx.x * per;
+  if (d >= N) return;
+  const int dend = min(d + per, N);
+  int lo = max(0, d - nb), hi = min(d, na);
+  while (lo < hi) {
+    const int mid = (lo + hi) >> 1;
+    if (zk[mid] <= wk[d - 1 - mid]) lo = mid + 1;
+    else hi = mid;
+  }
+  int i = lo, j = d - lo;
+  for (int o = d; o < dend; ++o) {
+    const bool takez = (j >= nb) || (i < na && zk[i] <= wk[j]);
+    u32 k, v = 0;
+    if (takez) { k = zk[i]; if (V) v = zv[i]; ++i; }
+    else { k = wk[j]; if (V) v = wv[j]; ++j; }
+    if (o < ma) { xk[o] = k; if (V) xv[o] = v; }
+    else { yk[o - ma] = k; if (V) yv[o - ma] = v; }
+  }
+}
+
+// Merge consecutive sorted runs of length `run` pairwise (src -> dst), n entries total,
+// n a multiple of 2*run.  Stable (earlier run first on ties).
+template <int NT, bool V>
+__device__ __forceinline__ void cta_merge_pass(const u32* __restrict__ sk, const u32* __restrict__ sv,
+                                               u32* __restrict__ dk, u32* __restrict__ dv, int n,
+                                               int run) {
+  const int per = (n + NT - 1) / NT;  // divides 2*run for the sizes used (powers of two)
+  const int d0 = threadIdx.x * per;
+  if (d0 >= n) return;
+  const int pair = d0 / (2 * run);
+  const int base = pair * 2 * run;
+  const u32* zk = sk + base;
+  const u32* wk = zk + run;
+  const u32* zv = V ? sv + base : nullptr;
+  const u32* wv = V ? zv + run : nullptr;
+  const int d = d0 - base;
+  int lo = max(0, d - run), hi = min(d, run);
+  while (lo < hi) {
+    const int mid = (lo + hi) >> 1;
+    if (zk[mid] <= wk[d - 1 - mid]) lo = mid + 1;
+    else hi = mid;
+  }
+  int i = lo, j = d - lo;
+  const int dend = min(d + per, 2 * run);
+  for (int o = d; o < dend; ++o) {
+    const bool takez = (j >= run) || (i < run && zk[i] <= wk[j]);
+    if (takez) { dk[base + o] = zk[i]; if (V) dv[base + o] = zv[i]; ++i; }
+    else { dk[base + o] = wk[j]; if (V) dv[base + o] = wv[j]; ++j; }
+  }
+}
+
+// Sort the first `s` entries of (k, v) (smem, capacity K >= 64, power of two).  Entries
+// [s, P) with P = max(64, next_pow2(s)) are treated as padding (sort after real entries).
+// Uses (t_k, t_v) as scratch; returns true if the sorted result ended up in the scratch.
+template <int K, int NT, bool V>
+__device__ __forceinline__ bool cta_sort(u32* k, u32* v, int s, u32* tk, u32* tv) {
+  int P = 64;
+  while (P < s) P <<= 1;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  for (int r = warp; r * 64 < P; r += NT / 32) {
+    const int e0 = r * 64 + lane, e1 = e0 + 32;
+    u64 c0 = ((u64)k[e0] << 1) | (u64)(e0 >= s);
+    u64 c1 = ((u64)k[e1] << 1) | (u64)(e1 >= s);
+    u32 v0 = 0, v1 = 0;
+    if (V) { v0 = v[e0]; v1 = v[e1]; }
+    warp_sort64<V>(c0, c1, v0, v1);
+    k[e0] = (u32)(c0 >> 1);
+    k[e1] = (u32)(c1 >> 1);
+    if (V) { v[e0] = v0; v[e1] = v1; }
+  }
+  __syncthreads();
+  bool in_scratch = false;
+  for (int run = 64; run < P; run <<= 1) {
+    if (!in_scratch) cta_merge_pass<NT, V>(k, v, tk, tv, P, run);
+    else cta_merge_pass<NT, V>(tk, tv, k, v, P, run);
+    in_scratch = !in_scratch;
+    __syncthreads();
+  }
+  return in_scratch;
+}
+
+}  // namespace bgpqd
