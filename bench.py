@@ -1,0 +1,337 @@
+#!/usr/bin/env python
+"""bench.py — BGPQ hot-path benchmark (BASELINE.json metric) on B200.
+
+Default workload (config C2, phased; BASELINE.json configs[1]): insert 2^27 uniform uint32
+keys into an empty BGPQ with K = 1024 (keys only, w = 4 B), then DELETEMIN all of them.
+One step = one pass of the whole hot path (all INSERT batches then all DELETEMIN batches).
+Metric: keys/s = keys / (t_insert + t_deletemin), device-timed with CUDA events.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+                    [--values] [--dist uniform|ascending|descending|gaussian] [--K 1024]
+                    [--n-log2 27] [--mix]
+
+Multi-GPU: the linearizable heap does not shard: N ranks run N independent
+replicas ("scaling": "weak"), timed as the max over ranks.
+--impl reference runs the CPU oracle (oracle/, std::multiset) on a bounded sample of the
+same workload on the host cores (rank 0 only).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "keys/sec insert & deletemin (128M keys, K=1024) on 1 B200; % HBM roofline"
+
+
+def _peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    return 6650.0, "fallback (B200_PROFILING.md: 6.65 TB/s)"
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled every 200 ms during the timed region."""
+    FIELDS = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,"
+              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+              "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.proc = None
+        self.lines: list[str] = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}",
+                 "--format=csv,noheader,nounits", "-lms", "200"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except FileNotFoundError:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.25)
+        self.proc.terminate()
+        self.proc.wait()
+        sm, smax, reasons = [], [], set()
+        names = ("hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap")
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 6:
+                continue
+            try:
+                sm.append(float(f[0])); smax.append(float(f[1]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[2:6]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        return {"sm_mhz": float(np.median(sm)) if sm else None,
+                "sm_max_mhz": max(smax) if smax else None,
+                "samples": len(sm), "reasons": sorted(reasons)}
+
+
+def byte_model(st: dict, K: int, w: int) -> dict:
+    """Algorithmic bytes of Alg.1-3, from device counters.
+    INSERT: K·w input read + 2K·w per intermediate path level + K·w target write.
+    DELETEMIN: K·w output + K·w read of the last node + 4K·w per heapify level + K·w final
+    write of the node the sinking keys stop in."""
+    ins = st["ins_ops"] * K * w + st["ins_levels"] * 2 * K * w + st["ins_heapify_ops"] * K * w
+    dele = st["keys_out"] * w + st["del_refill_ops"] * K * w + st["del_levels"] * 4 * K * w \
+        + st["del_refill_ops"] * K * w
+    skipped = st["ins_noop"] * 2 * K * w
+    return {"insert": ins, "deletemin": dele, "total": ins + dele, "insert_noop_skipped": skipped}
+
+
+def _dist_setup():
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return world, rank, local
+
+
+def run_reference(args, world, rank):
+    """CPU oracle (std::multiset, oracle/) on a bounded sample of the same workload."""
+    if rank != 0:
+        return
+    import oracle
+    import synth
+    oracle.build()
+    n_sample = 1 << args.ref_log2
+    keys = synth.keys(n_sample, seed=synth.SEEDS["C2"], dist=args.dist)
+    try:
+        os.sched_setaffinity(0, {sorted(os.sched_getaffinity(0))[0]})
+    except (AttributeError, OSError):
+        pass
+    times = []
+    for i in range(args.warmup + args.steps):
+        t0 = time.perf_counter()
+        out = oracle.pq_phased(keys, args.K)
+        dt = time.perf_counter() - t0
+        if i >= args.warmup:
+            times.append(dt)
+    assert np.array_equal(out[:1024], np.sort(keys)[:1024])
+    t = float(np.mean(times))
+    v = n_sample / t
+    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "keys/s", "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": t * 1e3, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+            "config": _config(args),
+            "cpu_baseline": {"value": v, "unit": "keys/s", "cores": 1, "kind": "oracle",
+                             "sample": f"phased insert-all/deletemin-all of 2^{args.ref_log2} keys "
+                                       f"(K={args.K}) through the std::multiset oracle, 1 pinned core"},
+            "e2e": {"value": v, "unit": "keys/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def _config(args):
+    w = 8 if args.values else 4
+    return {"workload": (f"C2 phased: insert 2^{args.n_log2} {args.dist} uint32 keys into an empty BGPQ "
+                         f"then deletemin all, K={args.K}, {'key+value' if args.values else 'keys only'} "
+                         f"(w={w} B)"),
+            "n_keys": 1 << args.n_log2, "K": args.K, "w_bytes": w, "dist": args.dist,
+            "threads_per_cta": 512, "l2": f"inputs and heap ({(1 << args.n_log2) * w * 3 >> 20} MiB) "
+                                          "larger than the 126 MB L2; no flush"}
+
+
+def cpu_baseline(args):
+    import oracle
+    import synth
+    oracle.build()
+    n_sample = 1 << args.ref_log2
+    keys = synth.keys(n_sample, seed=synth.SEEDS["C2"], dist=args.dist)
+    try:
+        os.sched_setaffinity(0, {sorted(os.sched_getaffinity(0))[0]})
+        cores = 1
+    except (AttributeError, OSError):
+        cores = 1
+    t0 = time.perf_counter()
+    out = oracle.pq_phased(keys, args.K)
+    dt = time.perf_counter() - t0
+    assert len(out) == n_sample
+    return {"value": n_sample / dt, "unit": "keys/s", "cores": cores, "kind": "oracle",
+            "sample": f"phased insert-all/deletemin-all of 2^{args.ref_log2} keys (K={args.K}), "
+                      f"std::multiset oracle, 1 pinned host core, {dt:.1f} s"}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--K", type=int, default=1024)
+    ap.add_argument("--n-log2", type=int, default=27)
+    ap.add_argument("--values", action="store_true")
+    ap.add_argument("--dist", default="uniform")
+    ap.add_argument("--ref-log2", type=int, default=22)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--profile-steps", type=int, default=0, help="ncu mode: run N untimed steps and exit")
+    args = ap.parse_args()
+    world, rank, local = _dist_setup()
+
+    if args.impl == "reference":
+        run_reference(args, world, rank)
+        return
+
+    import torch
+    import synth
+    import paper_conf_icpp_chenhjz21_b200 as pkg
+
+    torch.cuda.set_device(local)
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+
+    n, K = 1 << args.n_log2, args.K
+    w = 8 if args.values else 4
+    keys = synth.keys(n, seed=synth.SEEDS["C2"] + rank, dist=args.dist)
+    dk = torch.from_numpy(keys.view(np.int32)).cuda()
+    dv = torch.arange(n, dtype=torch.int32, device="cuda") if args.values else None
+    out_k = torch.empty(n, dtype=torch.int32, device="cuda")
+    out_v = torch.empty(n, dtype=torch.int32, device="cuda") if args.values else None
+    q = pkg.BGPQ(capacity=n, K=K, values=args.values)
+    stream = torch.cuda.current_stream()
+
+    def step(ev=None):
+        if ev: ev[0].record(stream)
+        q.insert(dk, dv, stream=stream)
+        if ev: ev[1].record(stream)
+        q.deletemin(n, out_k, out_v, stream=stream)
+        if ev: ev[2].record(stream)
+
+    if args.profile_steps:
+        for _ in range(args.profile_steps):
+            step()
+        torch.cuda.synchronize()
+        return
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    # parity spot check of the warm-up pass (full output vs sorted input, on device)
+    mask = 0xFFFFFFFF
+    ref_sorted = torch.sort(dk.to(torch.int64) & mask)[0]
+    ok_parity = bool(torch.equal(out_k.to(torch.int64) & mask, ref_sorted))
+    del ref_sorted
+
+    st0 = q.stats()
+    l0 = pkg.launch_count()
+    evs = [[torch.cuda.Event(enable_timing=True) for _ in range(3)] for _ in range(args.steps)]
+    clk = ClockSampler(local)
+    clk.start()
+    if dist: dist.barrier()
+    torch.cuda.synchronize()
+    t_start = torch.cuda.Event(enable_timing=True)
+    t_end = torch.cuda.Event(enable_timing=True)
+    t_start.record(stream)
+    for i in range(args.steps):
+        step(evs[i])
+    t_end.record(stream)
+    torch.cuda.synchronize()
+    if dist: dist.barrier()
+    clocks = clk.stop()
+    launches = pkg.launch_count() - l0
+    st1 = q.stats()
+    total_ms = t_start.elapsed_time(t_end)
+    ins_ms = [e[0].elapsed_time(e[1]) for e in evs]
+    del_ms = [e[1].elapsed_time(e[2]) for e in evs]
+    if dist:
+        t = torch.tensor([total_ms], device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        total_ms = float(t.item())
+    ms_per_step = total_ms / args.steps
+    value = world * n * args.steps / (total_ms / 1e3)
+
+    dst = {k: (st1[k] - st0[k]) // args.steps for k in st1}
+    bm = byte_model(dst, K, w)
+    peak, peak_src = _peaks()
+    del_s = float(np.mean(del_ms)) / 1e3
+    ins_s = float(np.mean(ins_ms)) / 1e3
+    achieved = bm["deletemin"] / del_s / 1e9
+    traffic = None
+    prof = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(prof):
+        try:
+            pj = json.load(open(prof))
+            key = f"K{K}_w{w}_n{args.n_log2}"
+            traffic = pj.get(key, {}).get("deletemin_dram_bytes")
+        except Exception:
+            traffic = None
+
+    e2e = None
+    if not args.no_e2e:
+        # public API with HOST buffers: H2D of the inputs and D2H of the results in the region
+        hk = torch.from_numpy(keys.view(np.int32)).pin_memory().numpy().view(np.uint32)
+        hv = np.arange(n, dtype=np.uint32) if args.values else None
+        if hv is not None:
+            hv = torch.from_numpy(hv.view(np.int32)).pin_memory().numpy().view(np.uint32)
+        ho = torch.empty(n, dtype=torch.int32).pin_memory().numpy().view(np.uint32)
+        hov = torch.empty(n, dtype=torch.int32).pin_memory().numpy().view(np.uint32) if args.values else None
+        q.insert_host(hk, hv)
+        q.deletemin_host(n, ho, hov)  # warm the staging buffers
+        e_steps = max(1, min(args.steps, 3))
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        for _ in range(e_steps):
+            q.insert_host(hk, hv)
+            cnt = q.deletemin_host(n, ho, hov)
+        torch.cuda.synchronize()
+        e_dt = (time.perf_counter() - t0) / e_steps
+        assert cnt == n
+        e2e = {"value": world * n / e_dt, "unit": "keys/s", "h2d_bytes_per_step": n * w,
+               "d2h_bytes_per_step": n * w + 8, "ms_per_step": e_dt * 1e3}
+
+    if rank == 0:
+        cpu = None if args.no_cpu_baseline else cpu_baseline(args)
+        line = {
+            "metric": METRIC, "value": value, "unit": "keys/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+            "config": _config(args),
+            "parallelism": "replicas only (one linearizable heap per GPU)",
+            "phases_ms": {"insert": float(np.mean(ins_ms)), "deletemin": float(np.mean(del_ms))},
+            "roofline": {"bound": "hbm", "kernel": "bgpq_ops_kernel (DELETEMIN launch)",
+                         "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+                         "traffic": traffic, "peak_source": peak_src,
+                         "alg_bytes_per_launch": bm["deletemin"]},
+            "roofline_step": {"alg_bytes_per_step": bm["total"],
+                              "achieved_GBps": bm["total"] / (ms_per_step / 1e3) / 1e9,
+                              "frac": bm["total"] / (ms_per_step / 1e3) / 1e9 / peak,
+                              "insert_GBps": bm["insert"] / ins_s / 1e9},
+            "counters_per_step": dst,
+            "gpu_launches": launches,
+            "clocks": clocks,
+            "e2e": e2e,
+            "cpu_baseline": cpu,
+            "parity_warmup_output_sorted": ok_parity,
+        }
+        print(json.dumps(line), flush=True)
+    if dist:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()
