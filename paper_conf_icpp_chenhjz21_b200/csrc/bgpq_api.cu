@@ -10,7 +10,7 @@
 #include <cstring>
 
 #include "../../include/bgpq.h"
-#include "bgpq_ops.cuh"
+#include "bgpq_server.cuh"
 
 using namespace bgpqd;
 
@@ -42,6 +42,9 @@ struct bgpq {
   int sm_count = 0;
   int occ = 0;         // co-resident CTAs per SM for this K
   int grid_req = 0;    // 0 auto, else exact
+  SrvArgs srv{};           // server-mode rings and control words (device)
+  bool srv_ok = false;
+  int srv_grid = 0;
   u32* stage_k = nullptr;  // staging for the *_host calls
   u32* stage_v = nullptr;
   u64* stage_cnt = nullptr;
@@ -68,6 +71,24 @@ struct KernelInfo {
     g_launches.fetch_add(1);
     return cudaGetLastError();
   }
+  static int srv_occupancy(int* out_occ) {
+    auto kern = bgpq_srv_kernel<K, V, NT>;
+    const size_t smem = SrvShape<K, V, NT>::smem;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return -1;
+    int occ = 0;
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, NT + 32, smem);
+    if (e != cudaSuccess) return -1;
+    *out_occ = occ;
+    return 0;
+  }
+  static cudaError_t srv_launch(int grid, const HeapArgs& H, const CallArgs& C, const SrvArgs& A,
+                                cudaStream_t s) {
+    bgpq_srv_kernel<K, V, NT><<<grid, NT + 32, SrvShape<K, V, NT>::smem, s>>>(H, C, A);
+    g_launches.fetch_add(1);
+    return cudaGetLastError();
+  }
+  static int srv_top_nodes() { return SrvShape<K, V, NT>::NTOP; }
 };
 
 int occupancy_for(u32 K, bool V, int* occ) {
@@ -102,6 +123,55 @@ cudaError_t launch_for(u32 K, bool V, int grid, const HeapArgs& H, const CallArg
 #undef BGPQ_CASE
 }
 
+int srv_occupancy_for(u32 K, bool V, int* occ) {
+#define BGPQ_CASE(KK)                                                                        \
+  case KK:                                                                                   \
+    return V ? KernelInfo<KK, true>::srv_occupancy(occ) : KernelInfo<KK, false>::srv_occupancy(occ);
+  switch (K) {
+    BGPQ_CASE(64)
+    BGPQ_CASE(128)
+    BGPQ_CASE(256)
+    BGPQ_CASE(512)
+    BGPQ_CASE(1024)
+    default:
+      return -1;
+  }
+#undef BGPQ_CASE
+}
+
+int srv_top_for(u32 K, bool V) {
+#define BGPQ_CASE(KK)                                                                        \
+  case KK:                                                                                   \
+    return V ? KernelInfo<KK, true>::srv_top_nodes() : KernelInfo<KK, false>::srv_top_nodes();
+  switch (K) {
+    BGPQ_CASE(64)
+    BGPQ_CASE(128)
+    BGPQ_CASE(256)
+    BGPQ_CASE(512)
+    BGPQ_CASE(1024)
+    default:
+      return 0;
+  }
+#undef BGPQ_CASE
+}
+
+cudaError_t srv_launch_for(u32 K, bool V, int grid, const HeapArgs& H, const CallArgs& C, const SrvArgs& A,
+                           cudaStream_t s) {
+#define BGPQ_CASE(KK)                                                                        \
+  case KK:                                                                                   \
+    return V ? KernelInfo<KK, true>::srv_launch(grid, H, C, A, s) : KernelInfo<KK, false>::srv_launch(grid, H, C, A, s);
+  switch (K) {
+    BGPQ_CASE(64)
+    BGPQ_CASE(128)
+    BGPQ_CASE(256)
+    BGPQ_CASE(512)
+    BGPQ_CASE(1024)
+    default:
+      return cudaErrorInvalidValue;
+  }
+#undef BGPQ_CASE
+}
+
 bool valid_K(u32 K) { return K == 64 || K == 128 || K == 256 || K == 512 || K == 1024; }
 
 HeapArgs heap_args(const bgpq* q) {
@@ -121,10 +191,24 @@ int grid_for(const bgpq* q, u64 n_ops) {
   return (int)std::max(1LL, g);
 }
 
+bool server_mode(const bgpq* q) { return !(q->flags & (BGPQ_FLAG_SERIAL | BGPQ_FLAG_LOCKS)); }
+
 int run_call(bgpq* q, const CallArgs& C, cudaStream_t s) {
+  const bool V = (q->flags & BGPQ_FLAG_VALUES) != 0;
+  if (server_mode(q)) {
+    // reset the per-call control words, publication flags, gate tickets and lend counters
+    const int ntop = srv_top_for(q->K, V);
+    bool ok = cudaMemsetAsync(q->srv.ctl, 0, C_WORDS * sizeof(u32), s) == cudaSuccess;
+    ok = ok && cudaMemsetAsync(q->srv.task_pub, 0, NTASK * sizeof(u32), s) == cudaSuccess;
+    ok = ok && cudaMemsetAsync(q->srv.sready, 0, NSB * sizeof(u32), s) == cudaSuccess;
+    ok = ok && cudaMemsetAsync(q->srv.serving, 0, ntop * sizeof(u32), s) == cudaSuccess;
+    ok = ok && cudaMemsetAsync(q->srv.ret, 0, ntop * sizeof(u32), s) == cudaSuccess;
+    if (!ok) return fail(BGPQ_ECUDA);
+    if (srv_launch_for(q->K, V, q->srv_grid, heap_args(q), C, q->srv, s) != cudaSuccess) return fail(BGPQ_ECUDA);
+    return BGPQ_OK;
+  }
   // reset the per-call ticket and fetch counter (header words H_CALL, H_FETCH)
   if (cudaMemsetAsync(q->hdr + H_CALL, 0, 2 * sizeof(u32), s) != cudaSuccess) return fail(BGPQ_ECUDA);
-  const bool V = (q->flags & BGPQ_FLAG_VALUES) != 0;
   if (launch_for(q->K, V, grid_for(q, C.n_ops), heap_args(q), C, s) != cudaSuccess) return fail(BGPQ_ECUDA);
   return BGPQ_OK;
 }
@@ -135,7 +219,7 @@ extern "C" {
 
 bgpq_t* bgpq_create_ex(uint64_t capacity, uint32_t K, uint32_t flags) {
   g_last_error = BGPQ_OK;
-  if (!valid_K(K) || capacity == 0 || (flags & ~3u)) {
+  if (!valid_K(K) || capacity == 0 || (flags & ~7u)) {
     fail(BGPQ_EINVAL);
     return nullptr;
   }
@@ -170,6 +254,35 @@ bgpq_t* bgpq_create_ex(uint64_t capacity, uint32_t K, uint32_t flags) {
   if (ok) ok = cudaMalloc(&q->hdr, HEADER_WORDS * sizeof(u32)) == cudaSuccess;
   if (ok) ok = cudaMemset(q->meta, 0, q->slots * sizeof(NodeMeta)) == cudaSuccess;
   if (ok) ok = cudaMemset(q->hdr, 0, HEADER_WORDS * sizeof(u32)) == cudaSuccess;
+  if (ok && server_mode(q)) {
+    int socc = 0;
+    if (srv_occupancy_for(K, V, &socc) != 0 || socc < 1) {
+      cudaDeviceSynchronize();
+      bgpq_destroy(q);
+      fail(BGPQ_ECUDA);
+      return nullptr;
+    }
+    q->srv_grid = q->sm_count * socc;  // every CTA co-resident: the server and all workers
+    const int ntop = srv_top_for(K, V);
+    SrvArgs& A = q->srv;
+    memset(&A, 0, sizeof(A));
+    const size_t kb = (size_t)K * sizeof(u32);
+    ok = cudaMalloc(&A.ctl, C_WORDS * sizeof(u32)) == cudaSuccess;
+    ok = ok && cudaMalloc(&A.task, (size_t)NTASK * 8 * sizeof(u32)) == cudaSuccess;
+    ok = ok && cudaMalloc(&A.task_pub, NTASK * sizeof(u32)) == cudaSuccess;
+    ok = ok && cudaMalloc(&A.payk, NTASK * kb) == cudaSuccess;
+    ok = ok && cudaMalloc(&A.sbk, NSB * kb) == cudaSuccess;
+    ok = ok && cudaMalloc(&A.sready, NSB * sizeof(u32)) == cudaSuccess;
+    ok = ok && cudaMalloc(&A.serving, ntop * sizeof(u32)) == cudaSuccess;
+    ok = ok && cudaMalloc(&A.ret, ntop * sizeof(u32)) == cudaSuccess;
+    ok = ok && cudaMalloc(&A.mailk, kb) == cudaSuccess;
+    if (V) {
+      ok = ok && cudaMalloc(&A.payv, NTASK * kb) == cudaSuccess;
+      ok = ok && cudaMalloc(&A.sbv, NSB * kb) == cudaSuccess;
+      ok = ok && cudaMalloc(&A.mailv, kb) == cudaSuccess;
+    }
+    q->srv_ok = ok;
+  }
   if (ok) ok = cudaDeviceSynchronize() == cudaSuccess;
   if (!ok) {
     cudaGetLastError();
@@ -192,6 +305,9 @@ void bgpq_destroy(bgpq_t* q) {
   cudaFree(q->stage_k);
   cudaFree(q->stage_v);
   cudaFree(q->stage_cnt);
+  SrvArgs& A = q->srv;
+  u32* bufs[] = {A.ctl, A.task, A.task_pub, A.payk, A.payv, A.sbk, A.sbv, A.sready, A.serving, A.ret, A.mailk, A.mailv};
+  for (u32* b : bufs) cudaFree(b);
   delete q;
 }
 
@@ -350,7 +466,7 @@ int bgpq_set_grid(bgpq_t* q, int ctas) {
   return BGPQ_OK;
 }
 
-int bgpq_grid(bgpq_t* q) { return q ? grid_for(q, ~0ull) : 0; }
+int bgpq_grid(bgpq_t* q) { return q ? (server_mode(q) ? q->srv_grid : grid_for(q, ~0ull)) : 0; }
 
 uint64_t bgpq_launch_count(void) { return g_launches.load(); }
 

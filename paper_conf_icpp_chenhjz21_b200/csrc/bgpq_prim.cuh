@@ -16,6 +16,8 @@ namespace bgpqd {
 typedef uint32_t u32;
 typedef uint64_t u64;
 typedef unsigned long long ull;
+typedef uint16_t u16;
+typedef uint8_t u8;
 
 constexpr u32 KEY_MAX = 0xFFFFFFFFu;
 
@@ -94,6 +96,11 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, u32 bytes, 
           smem_addr(dst)),
       "l"(src), "r"(bytes), "r"(smem_addr(bar)) : "memory");
 }
+
+// CTA barrier over the NT compute threads only (named barrier 1): the server CTA runs an
+// extra helper warp that must not take part in the compute barriers.
+template <int NT>
+__device__ __forceinline__ void cta_bar() { asm volatile("bar.sync 1, %0;" ::"n"(NT) : "memory"); }
 
 // ----------------------------------------------------------------------------------------
 // Sort(items) — Alg.1 l.2, bitonic sort [22].
@@ -174,6 +181,95 @@ __device__ __forceinline__ void cta_merge_split(const u32* __restrict__ zk, cons
   }
 }
 
+// ----------------------------------------------------------------------------------------
+// SORT_SPLIT by co-ranking every element (the final positions of a stable merge [11]):
+//   z[i] goes to i + #{w < z[i]},  w[j] goes to j + #{z <= w[j]}   (Z first on equal keys)
+// Each rank is a branchless fixed-trip binary search (no divergence); a thread handles up to
+// ceil(KMAX/NT) entries of each input so the independent searches overlap (ILP).  Output
+// position p < ma goes to X[p], else Y[p - ma].  X/Y must not alias Z/W.
+// ----------------------------------------------------------------------------------------
+__device__ __forceinline__ int lower_count(const u32* __restrict__ a, int n, u32 key, int top) {
+  // number of a[0:n) strictly below key; top = highest power of two <= max n (compile-time-ish)
+  int pos = 0;
+#pragma unroll
+  for (int step = top; step > 0; step >>= 1) {
+    const int q = pos + step;
+    if (q <= n && a[q - 1] < key) pos = q;
+  }
+  return pos;
+}
+__device__ __forceinline__ int upper_count(const u32* __restrict__ a, int n, u32 key, int top) {
+  int pos = 0;  // number of a[0:n) <= key
+#pragma unroll
+  for (int step = top; step > 0; step >>= 1) {
+    const int q = pos + step;
+    if (q <= n && a[q - 1] <= key) pos = q;
+  }
+  return pos;
+}
+template <int KMAX, int NT, bool V>
+__device__ __forceinline__ void cta_rank_merge(const u32* __restrict__ zk, const u32* __restrict__ zv,
+                                               int na, const u32* __restrict__ wk,
+                                               const u32* __restrict__ wv, int nb, int ma,
+                                               u32* __restrict__ xk, u32* __restrict__ xv,
+                                               u32* __restrict__ yk, u32* __restrict__ yv) {
+  constexpr int E = (KMAX + NT - 1) / NT;
+  u32 kz[E], kw[E];
+  int pz[E], pw[E];
+#pragma unroll
+  for (int e = 0; e < E; ++e) {
+    const int i = threadIdx.x + e * NT;
+    kz[e] = i < na ? zk[i] : 0u;
+    kw[e] = i < nb ? wk[i] : 0u;
+  }
+#pragma unroll
+  for (int e = 0; e < E; ++e) {
+    const int i = threadIdx.x + e * NT;
+    pz[e] = i + lower_count(wk, nb, kz[e], KMAX);
+    pw[e] = i + upper_count(zk, na, kw[e], KMAX);
+  }
+#pragma unroll
+  for (int e = 0; e < E; ++e) {
+    const int i = threadIdx.x + e * NT;
+    if (i < na) {
+      const int p = pz[e];
+      const u32 v = V ? zv[i] : 0u;
+      if (p < ma) { xk[p] = kz[e]; if (V) xv[p] = v; }
+      else { yk[p - ma] = kz[e]; if (V) yv[p - ma] = v; }
+    }
+    if (i < nb) {
+      const int p = pw[e];
+      const u32 v = V ? wv[i] : 0u;
+      if (p < ma) { xk[p] = kw[e]; if (V) xv[p] = v; }
+      else { yk[p - ma] = kw[e]; if (V) yv[p - ma] = v; }
+    }
+  }
+}
+
+// One pass of a bottom-up merge sort: merge sorted runs [2q*run, (2q+1)*run) and
+// [(2q+1)*run, (2q+2)*run) of src (n entries, n a multiple of 2*run) into dst, by co-ranking.
+template <int KMAX, int NT, bool V>
+__device__ __forceinline__ void cta_rank_merge_pass(const u32* __restrict__ sk, const u32* __restrict__ sv,
+                                                    u32* __restrict__ dk, u32* __restrict__ dv, int n,
+                                                    int run) {
+  constexpr int E = (KMAX + NT - 1) / NT;
+#pragma unroll
+  for (int e = 0; e < E; ++e) {
+    const int i = threadIdx.x + e * NT;
+    if (i < n) {
+      const u32 key = sk[i];
+      const int q = i / run;             // my run
+      const int base = (q & ~1) * run;   // start of the pair
+      const int off = i - q * run;       // index within my run
+      int p;
+      if ((q & 1) == 0) p = base + off + lower_count(sk + base + run, run, key, KMAX / 2);
+      else p = base + off + upper_count(sk + base, run, key, KMAX / 2);
+      dk[p] = key;
+      if (V) dv[p] = sv[i];
+    }
+  }
+}
+
 // Merge consecutive sorted runs of length `run` pairwise (src -> dst), n entries total,
 // n a multiple of 2*run.  Stable (earlier run first on ties).
 template <int NT, bool V>
@@ -224,13 +320,13 @@ __device__ __forceinline__ bool cta_sort(u32* k, u32* v, int s, u32* tk, u32* tv
     k[e1] = (u32)(c1 >> 1);
     if (V) { v[e0] = v0; v[e1] = v1; }
   }
-  __syncthreads();
+  cta_bar<NT>();
   bool in_scratch = false;
   for (int run = 64; run < P; run <<= 1) {
-    if (!in_scratch) cta_merge_pass<NT, V>(k, v, tk, tv, P, run);
-    else cta_merge_pass<NT, V>(tk, tv, k, v, P, run);
+    if (!in_scratch) cta_rank_merge_pass<K, NT, V>(k, v, tk, tv, P, run);
+    else cta_rank_merge_pass<K, NT, V>(tk, tv, k, v, P, run);
     in_scratch = !in_scratch;
-    __syncthreads();
+    cta_bar<NT>();
   }
   return in_scratch;
 }

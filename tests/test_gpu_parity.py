@@ -33,13 +33,19 @@ def _gpu_inv(q):
 # --------------------------------------------------------------------------------------
 # phased insert-all then deletemin-all: output == sorted(input) (closed form, §8(c))
 # --------------------------------------------------------------------------------------
+MODES = ["server", "locks"]
+
+
+@pytest.mark.parametrize("mode", MODES)
 @pytest.mark.parametrize("K", [64, 128, 256, 512, 1024])
 @pytest.mark.parametrize("dist", ["uniform", "ascending", "descending", "gaussian", "dups"])
-def test_phased_sorted(K, dist):
+def test_phased_sorted(K, dist, mode):
     n = 40 * K + 37  # several tiles and a ragged tail
+    if mode == "server":
+        n = 300 * K + 37  # deeper than the on-chip levels for every K
     keys = synth.keys(n, seed=synth.SEEDS["C3"], dist=dist)
     vals = synth.values(n)
-    q = pkg.BGPQ(capacity=n, K=K, values=True)
+    q = pkg.BGPQ(capacity=n, K=K, values=True, locks=(mode == "locks"))
     q.insert(_dev(keys), _dev(vals))
     assert q.size() == n
     assert _gpu_inv(q) == (0, 0)
@@ -166,9 +172,10 @@ def _replay_check(types, sizes, keys, in_off, outk, outv, cnt, lin, prefill=None
     return q
 
 
+@pytest.mark.parametrize("mode", MODES)
 @pytest.mark.parametrize("K,p_ins,partial", [(64, 0.5, True), (64, 0.5, False), (128, 0.55, True),
                                              (1024, 0.5, False)])
-def test_concurrent_mixed_replay(K, p_ins, partial):
+def test_concurrent_mixed_replay(K, p_ins, partial, mode):
     n_ops = 4000 if K <= 128 else 1200
     if partial:
         types, sizes = synth.random_ops(n_ops, K, seed=41 + K, p_insert=p_ins)
@@ -176,7 +183,7 @@ def test_concurrent_mixed_replay(K, p_ins, partial):
         types, _ = synth.random_ops(n_ops, K, seed=41 + K, p_insert=p_ins)
         sizes = np.full(n_ops, K, np.uint32)
     keys, in_off = _mixed_inputs(types, sizes, K, seed=43)
-    q = pkg.BGPQ(capacity=len(keys) + K, K=K, values=True)
+    q = pkg.BGPQ(capacity=len(keys) + K, K=K, values=True, locks=(mode == "locks"))
     outk, outv, cnt, lin = _run_mixed(q, types, sizes, keys, in_off)
     ref = _replay_check(types, sizes, keys, in_off, outk, outv, cnt, lin)
     for j in np.nonzero(types == 1)[0]:
@@ -188,11 +195,12 @@ def test_concurrent_mixed_replay(K, p_ins, partial):
     assert np.array_equal(_host(rest)[:len(rk)], rk)
 
 
-def test_concurrent_pairs_with_prefill_replay():
+@pytest.mark.parametrize("mode", MODES)
+def test_concurrent_pairs_with_prefill_replay(mode):
     """Utilisation shape: prefill, then insert/deletemin pairs on all CTAs."""
     K = 64
-    pre = synth.keys(1 << 14, seed=50)
-    q = pkg.BGPQ(capacity=(1 << 15) + 4096 * K, K=K, values=True)
+    pre = synth.keys(1 << 17, seed=50)
+    q = pkg.BGPQ(capacity=(1 << 18) + 4096 * K, K=K, values=True, locks=(mode == "locks"))
     q.insert(_dev(pre), _dev(synth.values(len(pre))))
     types, sizes = synth.mixed_ops(3000, K, seed=51, partial=True)
     keys, in_off = _mixed_inputs(types, sizes, K, seed=52)
@@ -201,7 +209,8 @@ def test_concurrent_pairs_with_prefill_replay():
     assert _gpu_inv(q) == (0, 0)
 
 
-def test_marked_handoff_replay():
+@pytest.mark.parametrize("mode", MODES)
+def test_marked_handoff_replay(mode):
     """Small heap, many concurrent full-batch inserts/deletemins: drives the TARGET/MARKED
     collaboration — the replay must stay exact whether or not it fires."""
     K = 64
@@ -210,7 +219,7 @@ def test_marked_handoff_replay():
         types, _ = synth.random_ops(3000, K, seed=60 + seed, p_insert=0.5)
         sizes = np.full(len(types), K, np.uint32)
         keys, in_off = _mixed_inputs(types, sizes, K, seed=70 + seed)
-        q = pkg.BGPQ(capacity=len(keys) + K, K=K, values=True)
+        q = pkg.BGPQ(capacity=len(keys) + K, K=K, values=True, locks=(mode == "locks"))
         outk, outv, cnt, lin = _run_mixed(q, types, sizes, keys, in_off)
         _replay_check(types, sizes, keys, in_off, outk, outv, cnt, lin)
         assert _gpu_inv(q) == (0, 0)
@@ -261,11 +270,12 @@ def test_host_api_roundtrip():
 # --------------------------------------------------------------------------------------
 # full size: config C2 (2^27 keys, K = 1024) in the launch configuration bench.py times
 # --------------------------------------------------------------------------------------
-def test_full_size_c2_properties():
+@pytest.mark.parametrize("mode", MODES)
+def test_full_size_c2_properties(mode):
     n, K = 1 << 27, 1024
     keys = synth.keys(n, seed=synth.SEEDS["C2"])
     dk = _dev(keys)
-    q = pkg.BGPQ(capacity=n, K=K, values=False)
+    q = pkg.BGPQ(capacity=n, K=K, values=False, locks=(mode == "locks"))
     q.insert(dk)
     assert q.size() == n
     ok, _ = q.deletemin(n)
