@@ -123,6 +123,7 @@ int bgpq_grid(bgpq_t* q);
 uint64_t bgpq_launch_count(void);
 
 int bgpq_last_error(void);
+const char* bgpq_last_error_msg(void); /* CUDA error string of the last BGPQ_ECUDA */
 const char* bgpq_strerror(int code);
 
 #ifdef __cplusplus

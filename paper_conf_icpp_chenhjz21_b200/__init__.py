@@ -80,6 +80,7 @@ def lib():
         L.bgpq_grid.argtypes = [_vp]
         L.bgpq_launch_count.restype = _u64
         L.bgpq_strerror.restype = ctypes.c_char_p
+        L.bgpq_last_error_msg.restype = ctypes.c_char_p
         _lib = L
     return _lib
 
@@ -88,7 +89,7 @@ def lib():
 EXPORTS = ("bgpq_create", "bgpq_create_ex", "bgpq_destroy", "bgpq_insert", "bgpq_deletemin",
            "bgpq_size", "bgpq_insert_host", "bgpq_deletemin_host", "bgpq_run_mixed", "bgpq_dump",
            "bgpq_slots", "bgpq_stats", "bgpq_set_grid", "bgpq_grid", "bgpq_launch_count",
-           "bgpq_last_error", "bgpq_strerror")
+           "bgpq_last_error", "bgpq_last_error_msg", "bgpq_strerror")
 
 
 class BGPQError(RuntimeError):
@@ -97,7 +98,8 @@ class BGPQError(RuntimeError):
 
 def _check(rc):
     if rc != BGPQ_OK:
-        raise BGPQError(f"bgpq error {rc}: {lib().bgpq_strerror(rc).decode()}")
+        msg = lib().bgpq_last_error_msg().decode() if rc == BGPQ_ECUDA else ""
+        raise BGPQError(f"bgpq error {rc}: {lib().bgpq_strerror(rc).decode()} {msg}")
 
 
 def _ptr(t):
@@ -139,7 +141,10 @@ class BGPQ:
 
     def close(self):
         if getattr(self, "_h", None):
-            lib().bgpq_destroy(self._h)
+            try:
+                lib().bgpq_destroy(self._h)
+            except Exception:  # interpreter shutdown
+                pass
             self._h = None
 
     __del__ = close

@@ -7,6 +7,7 @@
 #include <algorithm>
 #include <atomic>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 
 #include "../../include/bgpq.h"
@@ -19,10 +20,16 @@ namespace {
 constexpr int NT = 512;  // threads per CTA (the paper's block size)
 
 thread_local int g_last_error = BGPQ_OK;
+thread_local char g_last_msg[256] = "";
 std::atomic<unsigned long long> g_launches{0};
+unsigned g_debug = 0;  // test-only switches, from env BGPQ_DEBUG
 
 int fail(int code) {
   g_last_error = code;
+  if (code == BGPQ_ECUDA) {
+    cudaError_t e = cudaGetLastError();
+    snprintf(g_last_msg, sizeof(g_last_msg), "%s", cudaGetErrorString(e));
+  }
   return code;
 }
 
@@ -219,6 +226,7 @@ extern "C" {
 
 bgpq_t* bgpq_create_ex(uint64_t capacity, uint32_t K, uint32_t flags) {
   g_last_error = BGPQ_OK;
+  if (const char* d = getenv("BGPQ_DEBUG")) g_debug = (unsigned)atoi(d);
   if (!valid_K(K) || capacity == 0 || (flags & ~7u)) {
     fail(BGPQ_EINVAL);
     return nullptr;
@@ -322,6 +330,7 @@ int bgpq_insert(bgpq_t* q, const uint32_t* keys, const uint32_t* vals, uint64_t 
   C.n_ops = (n + q->K - 1) / q->K;
   C.in_k = keys;
   C.in_v = (q->flags & BGPQ_FLAG_VALUES) ? vals : nullptr;
+  C.debug = g_debug;
   return run_call(q, C, (cudaStream_t)stream);
 }
 
@@ -338,6 +347,7 @@ int bgpq_deletemin(bgpq_t* q, uint32_t* out_keys, uint32_t* out_vals, uint64_t n
   C.out_k = out_keys;
   C.out_v = (q->flags & BGPQ_FLAG_VALUES) ? out_vals : nullptr;
   C.d_count = reinterpret_cast<ull*>(d_count);
+  C.debug = g_debug;
   return run_call(q, C, (cudaStream_t)stream);
 }
 
@@ -360,6 +370,7 @@ int bgpq_run_mixed(bgpq_t* q, const uint8_t* op_types, const uint32_t* op_sizes,
   C.out_v = (q->flags & BGPQ_FLAG_VALUES) ? out_vals : nullptr;
   C.op_count = op_count;
   C.lin_ticket = reinterpret_cast<ull*>(lin_ticket);
+  C.debug = g_debug;
   return run_call(q, C, (cudaStream_t)stream);
 }
 
@@ -459,6 +470,13 @@ int bgpq_stats(bgpq_t* q, uint64_t* out, int n) {
   return BGPQ_OK;
 }
 
+int bgpq_debug_record(bgpq_t* q, uint32_t* out4) {
+  if (!q || !out4) return fail(BGPQ_EINVAL);
+  if (cudaDeviceSynchronize() != cudaSuccess) return fail(BGPQ_ECUDA);
+  if (cudaMemcpy(out4, q->hdr + 60, 16, cudaMemcpyDeviceToHost) != cudaSuccess) return fail(BGPQ_ECUDA);
+  return BGPQ_OK;
+}
+
 int bgpq_set_grid(bgpq_t* q, int ctas) {
   if (!q || ctas < 0) return fail(BGPQ_EINVAL);
   if (ctas > q->sm_count * q->occ) return fail(BGPQ_EINVAL);  // must stay co-resident
@@ -471,6 +489,7 @@ int bgpq_grid(bgpq_t* q) { return q ? (server_mode(q) ? q->srv_grid : grid_for(q
 uint64_t bgpq_launch_count(void) { return g_launches.load(); }
 
 int bgpq_last_error(void) { return g_last_error; }
+const char* bgpq_last_error_msg(void) { return g_last_msg; }
 
 const char* bgpq_strerror(int code) {
   switch (code) {

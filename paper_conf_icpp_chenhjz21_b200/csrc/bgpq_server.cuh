@@ -119,7 +119,7 @@ struct Server {
   u32* tmin;      // [NTOP]
   u32* tmax;      // [NTOP]
   volatile u32* tlent;  // [NTOP] 0 or 1 (set by main, cleared by the helper)
-  u32* texp;      // [NTOP] expected return sequence of a lent node
+  volatile u32* texp;  // [NTOP] expected return sequence of a lent node
   u32* tnext;     // [NTOP] gate ticket dispenser (gate g = GATE0 + i)
   u8* tav;        // [NTOP] AVAIL flag of on-chip nodes
   u32* sk;
@@ -191,10 +191,9 @@ struct Server {
   }
   // wait until an on-chip node is not lent to a worker (thread 0)
   __device__ __forceinline__ void wait_home(u32 n) {
-    if (n < (u32)NTOP && tlent[n]) {
-      u32 ns = 32;
-      while (ld_acquire_cta_shared(tlent + n)) { __nanosleep(ns); ns = ns < 512 ? ns * 2 : 512; }
-    }
+    if (n >= (u32)NTOP) return;
+    u32 ns = 32;
+    while (ld_acquire_cta_shared(tlent + n)) { __nanosleep(ns); ns = ns < 512 ? ns * 2 : 512; }
   }
 
   // ---- task publication (thread 0, after main_sync so payload stores are ordered)
@@ -358,6 +357,7 @@ struct Server {
     const u32 last_onchip = dt <= (u32)T ? dt - 1 : (u32)T;  // deepest on-chip path node depth
     for (u32 d = 1; d <= last_onchip; ++d) {
       const u32 c = tar >> (dt - d);
+      main_sync();
       if (tid == 0) {
         wait_home(c);
         const u32 cmin = tmin[c], cmax = tmax[c];
@@ -396,6 +396,7 @@ struct Server {
     }
     if (dt <= (u32)T) {  // l.9-10: target on chip
       if (tid == 0) {
+        release_slot(slot_of[tar]);  // every on-chip node keeps a slot; tar's was empty
         slot_of[tar] = (u16)it;
         tav[tar] = 1;
         tmin[tar] = imin; tmax[tar] = imax;
@@ -406,6 +407,7 @@ struct Server {
     // continuation below level T: INS_BODY task (gate g = ancestor of tar at depth T+1)
     const u32 g = tar >> (dt - (u32)(T + 1));
     u32 t = 0;
+    main_sync();
     if (tid == 0) {
       t = task_begin();
       sm->b[0] = t;
@@ -458,6 +460,7 @@ struct Server {
     }
     emit(ok, ov, 0, slot_of[1], 0, rs0);  // l.22
     nout = rs0;
+    main_sync();  // the root slot is read by every thread before thread 0 may swap it
     if (hs0 == 1) {  // l.23-29: refill from the buffer
       const u32 take = min(rs0 + ps0, size) - rs0;
       const int pb = slot_of[0];
@@ -521,6 +524,7 @@ struct Server {
     u32 cur = 1;
     bool stopped = false;
     for (;;) {
+      main_sync();  // thread 0's slot-table updates are visible; previous broadcast consumed
       const u32 dcur = depth_of(cur);
       if (dcur >= (u32)T) break;  // children are gate nodes: lend cur to a DEL_BODY task
       const u32 l = 2u * cur, r = l + 1u;
@@ -560,6 +564,7 @@ struct Server {
         }
       }
       // l.12: (Heap[cur], Heap[y]) <- SORT_SPLIT(Heap[cur], Heap[y])
+      main_sync();
       if (tid == 0) {
         const u32 swp = tmax[y] <= tmin[cur];
         if (swp) {
@@ -629,22 +634,57 @@ struct Server {
         const u32 tr = (r <= H.cap) ? tnext[r - GATE0]++ : 0u;
         const u32 seq = texp[cur] + 1u;
         texp[cur] = seq;
-        tlent[cur] = 1;
+        st_release_cta_shared(tlent + cur, 1u);  // texp before the lend flag (helper pairs them)
         const u32 t = task_begin();
         task_publish(t, TASK_DEL, cur, tl, tr, seq);
+        if (C.debug & 2u) wait_home(cur);
       }
     }
     if (tid == 0) *count_out = nout;
+    main_sync();
   }
 
   // ---- prefetch the refill node of the next op if it is a refilling DELETEMIN (thread 0)
   __device__ __forceinline__ void maybe_prefetch_tar(u64 jn) {
+    if (C.debug & 1u) return;
     if (jn >= C.n_ops || op_is_insert(jn)) return;
     if (hs < 2 || hs < (u32)NTOP) return;      // no refill, or the node is on chip
     if (op_size(jn) < rs) return;              // served from the root (Alg.2 l.18)
     if (sm->pf_node == hs) return;
     request_tar(hs);
     sm->pf_node = hs;
+  }
+
+  // debug (C.debug & 4): check the on-chip invariants after every operation (all main
+  // threads); the first violation is recorded in header words 60..63 {op+1, node, kind, hs}
+  __device__ void debug_check(u64 j) {
+    main_sync();
+    __shared__ u32 bad;
+    if (threadIdx.x == 0) bad = 0;
+    main_sync();
+    const u32 nn = min((u32)NTOP - 1, hs);
+    for (u32 i = 1; i <= nn; ++i) {
+      if (i >= 2 && (!tav[i] || tlent[i])) continue;
+      const u32 len = (i == 1) ? rs : (u32)K;
+      const u32* d = BK(slot_of[i]);
+      for (u32 e = threadIdx.x + 1; e < len; e += NT)
+        if (d[e - 1] > d[e]) atomicCAS(&bad, 0u, (i << 8) | 1u);
+      if (threadIdx.x == 0 && i >= 2) {
+        const u32 p = i / 2;
+        const bool pok = (p == 1) ? (rs == 0 || BK(slot_of[1])[rs - 1] <= d[0]) : (tlent[p] || BK(slot_of[p])[K - 1] <= d[0]);
+        if (!pok) atomicCAS(&bad, 0u, (i << 8) | 2u);
+        if (tmin[i] != d[0] || tmax[i] != d[K - 1]) atomicCAS(&bad, 0u, (i << 8) | 3u);
+      }
+    }
+    if (threadIdx.x == 0 && ps && rs && BK(slot_of[0])[0] < BK(slot_of[1])[rs - 1]) atomicCAS(&bad, 0u, 4u);
+    main_sync();
+    if (threadIdx.x == 0 && bad && ld_relaxed(H.hdr + 60) == 0) {
+      st_relaxed(H.hdr + 61, bad >> 8);
+      st_relaxed(H.hdr + 62, bad & 255u);
+      st_relaxed(H.hdr + 63, hs);
+      st_relaxed(H.hdr + 60, (u32)(j + 1));
+    }
+    main_sync();
   }
 
   __device__ void run() {
@@ -665,10 +705,11 @@ struct Server {
       tlent[i] = 0;
       texp[i] = 0;
       tnext[i] = 0;
-      const u32 sti = i >= 2 ? ld_relaxed(&H.meta[i].state) : 0u;
-      tav[i] = (i >= 2 && (u32)i <= H.cap && sti == ST_AVAIL) ? 1 : 0;
-      tmin[i] = ld_relaxed(&H.meta[i].kmin);
-      tmax[i] = ld_relaxed(&H.meta[i].kmax);
+      const bool ex = (u32)i <= H.cap;
+      const u32 sti = (i >= 2 && ex) ? ld_relaxed(&H.meta[i].state) : 0u;
+      tav[i] = (i >= 2 && ex && sti == ST_AVAIL) ? 1 : 0;
+      tmin[i] = ex ? ld_relaxed(&H.meta[i].kmin) : 0u;
+      tmax[i] = ex ? ld_relaxed(&H.meta[i].kmax) : 0u;
     }
     const u32 nload = min((u32)NTOP, H.cap + 1);
     for (u32 i = 0; i < nload; ++i) load_sync((int)i, H.gk + (size_t)i * K, V ? H.gv + (size_t)i * K : nullptr);
@@ -701,6 +742,7 @@ struct Server {
           maybe_prefetch_tar(j + 1);
         }
       }
+      if (C.debug & 4u) debug_check(j);
       if (tid == 0) {
         ++lin;
         st_relaxed(A.ctl + C_CONSUMED, (u32)(j + 1));
@@ -796,7 +838,7 @@ __device__ void helper_loop(Server<K, V, NT>& s) {
     }
     // (2) reload on-chip nodes returned by DEL_BODY workers
     for (int i = (1 << S::T); i < S::NTOP; ++i) {
-      if (!s.tlent[i]) continue;
+      if (!ld_acquire_cta_shared(s.tlent + i)) continue;
       if (ld_acquire(s.A.ret + i) != s.texp[i]) continue;
       idle = false;
       fence_proxy_async();
@@ -1161,7 +1203,7 @@ __global__ void __launch_bounds__(NT + 32, 1) bgpq_srv_kernel(HeapArgs H, CallAr
     s.tmin = reinterpret_cast<u32*>(p); p += 4 * S::NTOP;
     s.tmax = reinterpret_cast<u32*>(p); p += 4 * S::NTOP;
     s.tlent = reinterpret_cast<volatile u32*>(p); p += 4 * S::NTOP;
-    s.texp = reinterpret_cast<u32*>(p); p += 4 * S::NTOP;
+    s.texp = reinterpret_cast<volatile u32*>(p); p += 4 * S::NTOP;
     s.tnext = reinterpret_cast<u32*>(p); p += 4 * S::NTOP;
     s.tav = reinterpret_cast<u8*>(p); p += S::NTOP;
     s.sk = reinterpret_cast<u32*>(smem_raw + S::ctl_bytes);
