@@ -213,6 +213,18 @@ class BGPQ:
         _check(lib().bgpq_stats(self._h, out.ctypes.data_as(_vp), len(STAT_NAMES)))
         return dict(zip(STAT_NAMES, (int(x) for x in out)))
 
+    TIMER_NAMES = {0: "srv_total", 1: "srv_batch_wait", 2: "srv_tar_wait", 3: "srv_home_wait",
+                   4: "srv_task_wait", 5: "srv_merge", 6: "srv_ins", 7: "srv_del", 8: "srv_merges_n",
+                   16: "w_sort", 17: "w_ins", 18: "w_del", 19: "w_idle", 20: "w_ins_n", 21: "w_del_n",
+                   22: "w_sort_n", 9: "d_start", 10: "d_emit", 11: "d_refill", 12: "d_pb",
+                   13: "d_decide", 14: "d_lr", 15: "d_cy", 24: "d_extract", 25: "d_exit", 26: "d_lend"}
+
+    def timers(self) -> dict:
+        """Cycle counters of the server-mode kernel (cumulative; debug aid)."""
+        out = np.zeros(32, np.uint64)
+        _check(lib().bgpq_timers(self._h, out.ctypes.data_as(_vp)))
+        return {nm: int(out[i]) for i, nm in self.TIMER_NAMES.items()}
+
     def set_grid(self, ctas: int):
         _check(lib().bgpq_set_grid(self._h, int(ctas)))
 

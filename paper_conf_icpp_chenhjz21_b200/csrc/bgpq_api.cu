@@ -23,6 +23,7 @@ thread_local int g_last_error = BGPQ_OK;
 thread_local char g_last_msg[256] = "";
 std::atomic<unsigned long long> g_launches{0};
 unsigned g_debug = 0;  // test-only switches, from env BGPQ_DEBUG
+volatile u32* g_prog = nullptr;  // test-only progress log (host-mapped), bgpq_debug_progress()
 
 int fail(int code) {
   g_last_error = code;
@@ -331,6 +332,7 @@ int bgpq_insert(bgpq_t* q, const uint32_t* keys, const uint32_t* vals, uint64_t 
   C.in_k = keys;
   C.in_v = (q->flags & BGPQ_FLAG_VALUES) ? vals : nullptr;
   C.debug = g_debug;
+  C.prog = g_prog;
   return run_call(q, C, (cudaStream_t)stream);
 }
 
@@ -348,6 +350,7 @@ int bgpq_deletemin(bgpq_t* q, uint32_t* out_keys, uint32_t* out_vals, uint64_t n
   C.out_v = (q->flags & BGPQ_FLAG_VALUES) ? out_vals : nullptr;
   C.d_count = reinterpret_cast<ull*>(d_count);
   C.debug = g_debug;
+  C.prog = g_prog;
   return run_call(q, C, (cudaStream_t)stream);
 }
 
@@ -371,6 +374,7 @@ int bgpq_run_mixed(bgpq_t* q, const uint8_t* op_types, const uint32_t* op_sizes,
   C.op_count = op_count;
   C.lin_ticket = reinterpret_cast<ull*>(lin_ticket);
   C.debug = g_debug;
+  C.prog = g_prog;
   return run_call(q, C, (cudaStream_t)stream);
 }
 
@@ -467,6 +471,27 @@ int bgpq_stats(bgpq_t* q, uint64_t* out, int n) {
   ull st[NSTAT];
   if (cudaMemcpy(st, q->hdr + H_STAT, sizeof(st), cudaMemcpyDeviceToHost) != cudaSuccess) return fail(BGPQ_ECUDA);
   for (int i = 0; i < n && i < NSTAT; ++i) out[i] = st[i];
+  return BGPQ_OK;
+}
+
+// test-only: allocate (once) and return a 64-word host-mapped progress log
+uint32_t* bgpq_debug_progress(void) {
+  if (!g_prog) {
+    void* h = nullptr;
+    if (cudaHostAlloc(&h, 1024 * sizeof(u32), cudaHostAllocMapped) != cudaSuccess) return nullptr;
+    memset(h, 0, 1024 * sizeof(u32));
+    void* d = nullptr;
+    cudaHostGetDevicePointer(&d, h, 0);
+    g_prog = reinterpret_cast<volatile u32*>(d);
+    return reinterpret_cast<uint32_t*>(h);
+  }
+  return nullptr;
+}
+
+int bgpq_timers(bgpq_t* q, uint64_t* out32) {
+  if (!q || !out32) return fail(BGPQ_EINVAL);
+  if (cudaDeviceSynchronize() != cudaSuccess) return fail(BGPQ_ECUDA);
+  if (cudaMemcpy(out32, q->hdr + H_TIME, 32 * sizeof(u64), cudaMemcpyDeviceToHost) != cudaSuccess) return fail(BGPQ_ECUDA);
   return BGPQ_OK;
 }
 

@@ -59,20 +59,18 @@ __device__ __forceinline__ void fence_proxy_async() {
 // Node lock (D4): test-and-test-and-set with an acquire CAS; one elected thread spins
 // with __nanosleep backoff so the CAS traffic does not starve the holder's accesses.
 __device__ __forceinline__ u32 lock_acquire(u32* lk) {
-  u32 spins = 0, ns = 32;
+  u32 spins = 0, ns = 16;
   for (;;) {
     if (ld_relaxed(lk) == 0u && cas_acquire(lk, 0u, 1u) == 0u) return spins;
     ++spins;
     __nanosleep(ns);
-    ns = ns < 256 ? ns * 2 : 256;
+    ns = ns < 128 ? ns * 2 : 128;
   }
 }
 // Release: the caller has made all of the CTA's writes to the protected data happen-before
-// this thread (by __syncthreads); the gpu-scope fence + release store publishes them.
-__device__ __forceinline__ void lock_release(u32* lk) {
-  __threadfence();
-  st_release(lk, 0u);
-}
+// this thread with a CTA barrier (bar.sync is morally strong and orders them before this
+// thread's later accesses); the gpu-scope release store is cumulative and publishes them.
+__device__ __forceinline__ void lock_release(u32* lk) { st_release(lk, 0u); }
 
 // mbarrier + TMA bulk copy (global -> shared), completion by transaction bytes.
 __device__ __forceinline__ void mbar_init(u64* bar, u32 count) {
@@ -242,6 +240,79 @@ __device__ __forceinline__ void cta_rank_merge(const u32* __restrict__ zk, const
       const u32 v = V ? wv[i] : 0u;
       if (p < ma) { xk[p] = kw[e]; if (V) xv[p] = v; }
       else { yk[p - ma] = kw[e]; if (V) yv[p - ma] = v; }
+    }
+  }
+}
+
+// ----------------------------------------------------------------------------------------
+// SORT_SPLIT by merge path [11] with register windows (the hot-path merge).
+// Thread t produces the VT = ceil(2*KMAX/NT) consecutive outputs [t*VT, t*VT+VT) of the
+// stable merge (Z before W on equal keys): one fixed-trip branchless co-rank search on its
+// start diagonal, a serial merge of VT entries in registers, then vector stores (128-bit
+// when VT = 4).  Values are gathered after the key merge from the recorded source index.
+// Output position p < ma goes to X[p], else Y[p - ma].  X/Y must not alias Z/W.
+// ----------------------------------------------------------------------------------------
+template <int N>
+struct Log2Ceil { static constexpr int v = (N <= 1) ? 0 : 1 + Log2Ceil<(N + 1) / 2>::v; };
+template <>
+struct Log2Ceil<1> { static constexpr int v = 0; };
+
+template <int KMAX, int NT, bool V>
+__device__ __forceinline__ void cta_path_merge(const u32* __restrict__ zk, const u32* __restrict__ zv,
+                                               int na, const u32* __restrict__ wk,
+                                               const u32* __restrict__ wv, int nb, int ma,
+                                               u32* __restrict__ xk, u32* __restrict__ xv,
+                                               u32* __restrict__ yk, u32* __restrict__ yv) {
+  constexpr int VT = (2 * KMAX + NT - 1) / NT;
+  constexpr int LOG = Log2Ceil<KMAX + 1>::v;
+  const int N = na + nb;
+  const int d = threadIdx.x * VT;
+  if (d >= N) return;
+  int lo = max(0, d - nb), hi = min(d, na);
+#pragma unroll
+  for (int it = 0; it < LOG; ++it) {
+    const int len = hi - lo;
+    const int mid = lo + (len >> 1);
+    const bool act = len > 0;
+    const u32 a = zk[act ? mid : 0];
+    const u32 b = wk[act ? d - 1 - mid : 0];
+    const bool right = act && (a <= b);
+    lo = right ? mid + 1 : lo;
+    hi = (act && !right) ? mid : hi;
+  }
+  int i = lo, j = d - lo;
+  u32 a = (i < na) ? zk[i] : 0u;
+  u32 b = (j < nb) ? wk[j] : 0u;
+  u32 ko[VT];
+  int src[VT];
+#pragma unroll
+  for (int k = 0; k < VT; ++k) {
+    const bool takez = (j >= nb) || (i < na && a <= b);
+    ko[k] = takez ? a : b;
+    src[k] = takez ? i : (KMAX + j);
+    if (takez) { ++i; a = (i < na) ? zk[i] : 0u; }
+    else { ++j; b = (j < nb) ? wk[j] : 0u; }
+  }
+  u32 vo[VT];
+  if (V) {
+#pragma unroll
+    for (int k = 0; k < VT; ++k) vo[k] = src[k] < KMAX ? zv[src[k]] : wv[src[k] - KMAX];
+  }
+  if (VT == 4 && d + 4 <= N && ((d + 4 <= ma) || (d >= ma && ((ma & 3) == 0)))) {
+    u32* dk = (d + 4 <= ma) ? xk + d : yk + (d - ma);
+    *reinterpret_cast<uint4*>(dk) = make_uint4(ko[0], ko[1 % VT], ko[2 % VT], ko[3 % VT]);
+    if (V) {
+      u32* dv = (d + 4 <= ma) ? xv + d : yv + (d - ma);
+      *reinterpret_cast<uint4*>(dv) = make_uint4(vo[0], vo[1 % VT], vo[2 % VT], vo[3 % VT]);
+    }
+  } else {
+#pragma unroll
+    for (int k = 0; k < VT; ++k) {
+      const int o = d + k;
+      if (o < N) {
+        if (o < ma) { xk[o] = ko[k]; if (V) xv[o] = vo[k]; }
+        else { yk[o - ma] = ko[k]; if (V) yv[o - ma] = vo[k]; }
+      }
     }
   }
 }

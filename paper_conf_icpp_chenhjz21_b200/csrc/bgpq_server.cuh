@@ -43,13 +43,21 @@ constexpr int srv_depth() {
 }
 
 enum : u32 { TASK_INS = 1, TASK_DEL = 2 };
+// cycle counters (header words H_TIME..): server thread 0 and worker thread 0 sums
+enum : int {
+  TM_SRV_TOTAL = 0, TM_SRV_BATCH_WAIT, TM_SRV_TAR_WAIT, TM_SRV_HOME_WAIT, TM_SRV_TASK_WAIT,
+  TM_SRV_MERGE, TM_SRV_INS, TM_SRV_DEL, TM_SRV_MERGES_N,
+  TM_W_SORT = 16, TM_W_INS, TM_W_DEL, TM_W_IDLE, TM_W_INS_N, TM_W_DEL_N, TM_W_SORT_N, TM_W_LOCKWAIT,
+  TM_N = 32
+};
 constexpr u32 NTASK = 8192;  // task ring
 constexpr u32 NSB = 1024;    // sorted-batch ring
 
 // per-call control words (reset by the host before each call)
+// (each word on its own 128-B line: the workers poll some of them)
 enum : int {
-  C_TASK_HEAD = 0, C_TASK_TAIL = 1, C_SORT_NEXT = 2, C_CONSUMED = 3, C_DONE = 4, C_MAIL = 5,
-  C_WORDS = 8
+  C_TASK_HEAD = 0, C_TASK_TAIL = 32, C_SORT_NEXT = 64, C_CONSUMED = 96, C_DONE = 128, C_MAIL = 160,
+  C_WORDS = 192
 };
 
 struct SrvArgs {
@@ -127,12 +135,19 @@ struct Server {
   u32 phase_main, phase_b[2];
   // thread-0 state
   u32 hs, rs, ps;
+  u32 tail;  // next task index (only the server publishes tasks)
   ull lin;
   ull st[NSTAT];
+  ull tm[TM_N];
 
   __device__ __forceinline__ u32* BK(int s) const { return sk + s * K; }
   __device__ __forceinline__ u32* BV(int s) const { return V ? sv + s * K : nullptr; }
   __device__ __forceinline__ bool is_gate(u32 n) const { return n >= (u32)GATE0 && n < 2u * GATE0; }
+
+  ull tmark;
+  __device__ __forceinline__ void sec(int id) {  // thread 0: cycles since the previous mark -> tm[id]
+    if (threadIdx.x == 0) { const ull t = clock64(); tm[id] += t - tmark; tmark = t; }
+  }
 
   __device__ __forceinline__ int alloc() {  // thread 0
     const u32 n = sm->nfree;
@@ -180,8 +195,10 @@ struct Server {
   }
   __device__ __forceinline__ void merge(int z, int na, int w, int nb, int ma, int x, int y) {
     main_sync();
+    const ull t0 = clock64();
     cta_rank_merge<K, NT, V>(BK(z), BV(z), na, BK(w), BV(w), nb, ma, BK(x), BV(x), BK(y), BV(y));
     main_sync();
+    if (threadIdx.x == 0) { tm[TM_SRV_MERGE] += clock64() - t0; tm[TM_SRV_MERGES_N]++; }
   }
   __device__ __forceinline__ void emit(u32* ok, u32* ov, u32 pos, int s, int off, int n) {
     for (int i = threadIdx.x; i < n; i += NT) {
@@ -192,15 +209,21 @@ struct Server {
   // wait until an on-chip node is not lent to a worker (thread 0)
   __device__ __forceinline__ void wait_home(u32 n) {
     if (n >= (u32)NTOP) return;
+    if (!ld_acquire_cta_shared(tlent + n)) return;
+    const ull t0 = clock64();
     u32 ns = 32;
     while (ld_acquire_cta_shared(tlent + n)) { __nanosleep(ns); ns = ns < 512 ? ns * 2 : 512; }
+    tm[TM_SRV_HOME_WAIT] += clock64() - t0;
   }
 
   // ---- task publication (thread 0, after main_sync so payload stores are ordered)
   __device__ __forceinline__ u32 task_begin() {
-    const u32 t = ld_relaxed(A.ctl + C_TASK_TAIL);
+    const u32 t = tail;
     if (t >= NTASK) {  // ring slot reuse: the task NTASK earlier must have been claimed+copied
+      const ull t0 = clock64();
+      if (C.prog) C.prog[1] = 4;
       while (ld_acquire(A.task_pub + (t % NTASK)) != 0xFFFFFFFFu - (t - NTASK)) __nanosleep(64);
+      tm[TM_SRV_TASK_WAIT] += clock64() - t0;
     }
     return t;
   }
@@ -211,9 +234,9 @@ struct Server {
     st_relaxed(d + 2, a1);
     st_relaxed(d + 3, a2);
     st_relaxed(d + 4, a3);
-    __threadfence();
     st_release(A.task_pub + (t % NTASK), t + 1);
     st_release(A.ctl + C_TASK_TAIL, t + 1);
+    tail = t + 1;
   }
 
   // ---- op descriptors
@@ -259,12 +282,22 @@ struct Server {
     const int b = (int)(j & 1);
     // the sorted batch (Alg.1 l.2 done by a worker before the root section)
     if (tid == 0) {
+      const ull t0 = clock64();
+      if (C.prog) C.prog[1] = 1;
       while (!try_prefetch_batch(j, issued)) __nanosleep(64);
+      if (C.prog) C.prog[1] = 2;
+      tm[TM_SRV_BATCH_WAIT] += clock64() - t0;
       if (*issued < j + 2) try_prefetch_batch(j + 1, issued);
       st[S_INS_OPS]++;
     }
     main_sync();
-    mbar_wait(&sm->bar_b[b], phase_b[b]);
+    {
+      const ull t0 = clock64();
+      if (tid == 0 && C.prog) C.prog[2] = (u32)(*issued);
+      mbar_wait(&sm->bar_b[b], phase_b[b]);
+      if (tid == 0 && C.prog) C.prog[1] = 3;
+      if (tid == 0) tm[TM_SRV_BATCH_WAIT] += clock64() - t0;
+    }
     phase_b[b] ^= 1u;
     if (tid == 0) {
       sm->b[0] = alloc();
@@ -430,6 +463,7 @@ struct Server {
   __device__ void do_deletemin(u64 j, u32 size, u32* ok, u32* ov, u32* count_out) {
     // (the refill node of op j+1 is requested as soon as |root| and heapSize are final)
     const int tid = threadIdx.x;
+    if (tid == 0) tmark = clock64();
     if (tid == 0) {
       st[S_DEL_OPS]++;
       sm->b[0] = hs; sm->b[1] = rs; sm->b[2] = ps;
@@ -437,6 +471,7 @@ struct Server {
     main_sync();
     const u32 hs0 = sm->b[0], rs0 = sm->b[1], ps0 = sm->b[2];
     u32 nout = 0;
+    sec(9);
     if (hs0 == 0) {  // l.16-17
       if (tid == 0) *count_out = 0;
       return;
@@ -461,6 +496,7 @@ struct Server {
     emit(ok, ov, 0, slot_of[1], 0, rs0);  // l.22
     nout = rs0;
     main_sync();  // the root slot is read by every thread before thread 0 may swap it
+    sec(10);
     if (hs0 == 1) {  // l.23-29: refill from the buffer
       const u32 take = min(rs0 + ps0, size) - rs0;
       const int pb = slot_of[0];
@@ -493,7 +529,9 @@ struct Server {
         sm->b[3] = 0;
       } else {  // taken by the helper under tar's lock (normally prefetched)
         if (sm->pf_node != tar) request_tar(tar);
+        const ull t0 = clock64();
         while (ld_acquire_cta_shared(&sm->tar_done) != sm->tar_req) __nanosleep(32);
+        tm[TM_SRV_TAR_WAIT] += clock64() - t0;
         if (sm->tar_marked) st[S_MARKED]++;
         sm->b[3] = 1;
       }
@@ -502,6 +540,7 @@ struct Server {
     main_sync();
     if (sm->b[3]) copy_slot(slot_of[1], S::S_TAR, 0, K);
     if (tid == 0) { tmin[1] = BK(slot_of[1])[0]; tmax[1] = BK(slot_of[1])[K - 1]; }
+    sec(11);
     // l.13: (root, pBuffer) <- SORT_SPLIT(root, K, pBuffer, |pB|, K)
     if (ps0 > 0) {
       if (tid == 0) {
@@ -520,6 +559,7 @@ struct Server {
         }
       }
     }
+    sec(12);
     // ---- l.14: DELETEMIN_HEAPIFY on chip (cur at depth < T: children on chip)
     u32 cur = 1;
     bool stopped = false;
@@ -551,6 +591,7 @@ struct Server {
         sm->b[6] = slot_of[l]; sm->b[7] = slot_of[r];
       }
       main_sync();
+      sec(13);
       const u32 stop = sm->b[0], x = sm->b[1], y = sm->b[2], lr = sm->b[3];
       if (stop) { stopped = true; break; }
       if (lr == 2) {  // l.10: (Heap[y], Heap[x]) <- SORT_SPLIT(Heap[l], Heap[r])
@@ -565,6 +606,7 @@ struct Server {
       }
       // l.12: (Heap[cur], Heap[y]) <- SORT_SPLIT(Heap[cur], Heap[y])
       main_sync();
+      sec(14);
       if (tid == 0) {
         const u32 swp = tmax[y] <= tmin[cur];
         if (swp) {
@@ -588,6 +630,7 @@ struct Server {
           tmin[y] = BK(c)[0]; tmax[y] = BK(c)[K - 1];
         }
       }
+      sec(15);
       if (cur == 1) {  // l.13: EXTRACT_ROOT(items, remainedSize)
         main_sync();
         const int rsl = slot_of[1];
@@ -605,8 +648,10 @@ struct Server {
           maybe_prefetch_tar(j + 1);
         }
       }
+      sec(16);
       cur = y;  // l.15
     }
+    sec(17);
     if (stopped) {
       if (cur == 1) {  // l.5-6
         main_sync();
@@ -640,6 +685,7 @@ struct Server {
         if (C.debug & 2u) wait_home(cur);
       }
     }
+    sec(18);
     if (tid == 0) *count_out = nout;
     main_sync();
   }
@@ -698,6 +744,10 @@ struct Server {
       asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(H.hdr + H_LIN) : "memory");
       lin = v;
       for (int i = 0; i < NSTAT; ++i) st[i] = 0;
+      for (int i = 0; i < TM_N; ++i) tm[i] = 0;
+      tm[31] = clock64();
+      tail = 0;
+      tmark = 0;
       sm->pf_node = 0xFFFFFFFFu;
     }
     for (int i = tid; i < NTOP; i += NT) {
@@ -720,10 +770,11 @@ struct Server {
     for (u64 j = 0; j < C.n_ops; ++j) {
       const u32 size = op_size(j);
       if (tid == 0 && C.mode == MODE_MIXED && C.lin_ticket) C.lin_ticket[j] = lin;
+      const ull top0 = clock64();
+      if (tid == 0 && C.prog) { C.prog[0] = (u32)j; C.prog[1] = 0; }
       if (op_is_insert(j)) {
-        const u64 off = C.mode == MODE_MIXED ? C.in_off[j] : j * (u64)K;
-        (void)off;
         do_insert(j, size, &issued);
+        if (tid == 0) tm[TM_SRV_INS] += clock64() - top0;
       } else {
         u32* ok = C.out_k;
         u32* ov = C.out_v;
@@ -736,6 +787,7 @@ struct Server {
         main_sync();
         cnt = sm->b[20];
         if (tid == 0) {
+          tm[TM_SRV_DEL] += clock64() - top0;
           st[S_KEYS_OUT] += cnt;
           if (C.mode == MODE_MIXED) C.op_count[j] = cnt;
           if (C.d_count && cnt) atomicAdd(C.d_count, (ull)cnt);
@@ -752,6 +804,7 @@ struct Server {
       main_sync();
     }
     // ---- end of call: wait for lent nodes, write the on-chip state back, stop helper
+    if (tid == 0 && C.prog) C.prog[1] = 10;
     if (tid == 0) {
       for (int i = 2; i < NTOP; ++i) wait_home((u32)i);
       st_release(A.ctl + C_DONE, 1u);
@@ -776,7 +829,13 @@ struct Server {
       asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(H.hdr + H_LIN), "l"(lin) : "memory");
       ull* stat = reinterpret_cast<ull*>(H.hdr + H_STAT);
       for (int i = 0; i < NSTAT; ++i) if (st[i]) atomicAdd(stat + i, st[i]);
+      tm[TM_SRV_TOTAL] = clock64() - tm[31];
+      tm[31] = 0;
+      ull* tms = reinterpret_cast<ull*>(H.hdr + H_TIME);
+      for (int i = 0; i < 9; ++i) if (tm[i]) atomicAdd(tms + i, tm[i]);
+      for (int i = 9; i <= 18; ++i) if (tm[i]) atomicAdd(tms + (i < 16 ? i : i + 8), tm[i]);
       sm->stop = 1;
+      if (C.prog) C.prog[1] = 11;
     }
   }
 };
@@ -795,8 +854,8 @@ __device__ void helper_loop(Server<K, V, NT>& s) {
   for (;;) {
     bool idle = true;
     // (1) refill node of the next DELETEMIN (Alg.2 l.6-12, taken under its lock)
-    const u32 req = ld_acquire_cta_shared(&s.sm->tar_req);
-    if (req != done) {
+    if (s.sm->tar_req != done) {
+      const u32 req = ld_acquire_cta_shared(&s.sm->tar_req);
       idle = false;
       const u32 n = s.sm->tar_node, ticket = s.sm->tar_ticket;
       const bool gate = s.is_gate(n);
@@ -811,7 +870,7 @@ __device__ void helper_loop(Server<K, V, NT>& s) {
       u32 marked = 0;
       if (state == ST_TARGET) {  // l.7-9: steal the keys of the insert in flight
         st_relaxed(&s.H.meta[n].state, ST_MARKED);
-        if (gate) { __threadfence(); st_release(s.A.serving + (n - S::GATE0), ticket + 1); }
+        if (gate) st_release(s.A.serving + (n - S::GATE0), ticket + 1);
         else lock_release(&s.H.meta[n].lock);
         while (ld_acquire(s.A.ctl + C_MAIL) == mail_seen) __nanosleep(64);
         mail_seen++;
@@ -829,7 +888,7 @@ __device__ void helper_loop(Server<K, V, NT>& s) {
         mbar_wait(&s.sm->bar_help, phase);
         phase ^= 1u;
         st_relaxed(&s.H.meta[n].state, ST_EMPTY);
-        if (gate) { __threadfence(); st_release(s.A.serving + (n - S::GATE0), ticket + 1); }
+        if (gate) st_release(s.A.serving + (n - S::GATE0), ticket + 1);
         else lock_release(&s.H.meta[n].lock);
       }
       s.sm->tar_marked = marked;
@@ -838,6 +897,7 @@ __device__ void helper_loop(Server<K, V, NT>& s) {
     }
     // (2) reload on-chip nodes returned by DEL_BODY workers
     for (int i = (1 << S::T); i < S::NTOP; ++i) {
+      if (!s.tlent[i]) continue;  // plain scan; acquire only on a hit
       if (!ld_acquire_cta_shared(s.tlent + i)) continue;
       if (ld_acquire(s.A.ret + i) != s.texp[i]) continue;
       idle = false;
@@ -854,7 +914,7 @@ __device__ void helper_loop(Server<K, V, NT>& s) {
       st_release_cta_shared(s.tlent + i, 0u);
     }
     if (s.sm->stop) break;
-    if (idle) __nanosleep(32);
+    if (idle) __nanosleep(64);
   }
 }
 
@@ -869,6 +929,7 @@ struct Worker {
   SrvArgs A;
   CallArgs C;
   Op<K, V, NT> op;  // smem slots / load / store / merge helpers (6 slots)
+  ull tm[8];
 
   __device__ __forceinline__ bool is_gate(u32 n) const { return n >= (u32)GATE0 && n < 2u * GATE0; }
   __device__ __forceinline__ void acquire(u32 n, u32 ticket) {  // thread 0
@@ -881,7 +942,7 @@ struct Worker {
     fence_proxy_async();
   }
   __device__ __forceinline__ void release(u32 n, u32 ticket) {  // thread 0
-    if (is_gate(n)) { __threadfence(); st_release(A.serving + (n - GATE0), ticket + 1); }
+    if (is_gate(n)) st_release(A.serving + (n - GATE0), ticket + 1);
     else lock_release(&H.meta[n].lock);
   }
 
@@ -910,7 +971,7 @@ struct Worker {
       for (int i = tid; i < K / 4; i += NT) dv[i] = sv4[i];
     }
     cta_bar<NT>();
-    if (tid == 0) { __threadfence(); st_release(A.sready + s, (u32)(j + 1)); }
+    if (tid == 0) st_release(A.sready + s, (u32)(j + 1));
   }
 
   // ---- INS_BODY: INSERT_HEAPIFY from gate node g (held via its ticket) to tar
@@ -933,7 +994,9 @@ struct Worker {
     if (tid == 0) {  // payload copied: the ring slot may be reused
       __threadfence();
       st_release(A.task_pub + (task % NTASK), 0xFFFFFFFFu - task);
+      if (C.prog) C.prog[17 + 2 * blockIdx.x] = 1;
       acquire(g, ticket);  // LOCK(g): gate tickets keep the server's order
+      if (C.prog) C.prog[17 + 2 * blockIdx.x] = 2;
     }
     cta_bar<NT>();
     u32 imin = op.BK(it)[0], imax = op.BK(it)[K - 1];
@@ -947,6 +1010,7 @@ struct Worker {
         u32 dec = 0, cmin = 0, cmax = 0;
         if (!brk) {
           if (!first) {  // l.32: LOCK(cur); UNLOCK(PARENT(cur))
+            if (C.prog) C.prog[17 + 2 * blockIdx.x] = 0x100000 | c;
             acquire(c, 0);
             release(held, held_ticket);
           }
@@ -985,6 +1049,7 @@ struct Worker {
     cta_bar<NT>();
     if (tid == 0) {
       if (tar != held) {
+        if (C.prog) C.prog[17 + 2 * blockIdx.x] = 0x200000 | tar;
         acquire(tar, 0);  // tar lies below the gate node: an ordinary node lock
         release(held, held_ticket);
       } else {
@@ -994,6 +1059,7 @@ struct Worker {
     }
     cta_bar<NT>();
     const u32 tar_ticket = (tar == held) ? held_ticket : 0u;
+    if (tid == 0 && C.prog) C.prog[17 + 2 * blockIdx.x] = 0x300000 | op.ctl->b[0];
     if (op.ctl->b[0] == ST_TARGET) {  // l.9-10
       op.store(tar, it);
       if (tid == 0) {
@@ -1027,7 +1093,7 @@ struct Worker {
     const int tid = threadIdx.x;
     const u32* d = A.task + (size_t)(task % NTASK) * 8;
     const u32 y0 = ld_relaxed(d + 1), tl0 = ld_relaxed(d + 2), tr0 = ld_relaxed(d + 3), seq = ld_relaxed(d + 4);
-    if (tid == 0) { __threadfence(); st_release(A.task_pub + (task % NTASK), 0xFFFFFFFFu - task); }
+    if (tid == 0) st_release(A.task_pub + (task % NTASK), 0xFFFFFFFFu - task);
     int R = 0;
     op.load(R, y0);  // the sinking keys the server left in y's global slot
     u32 cur = y0, cur_ticket = 0;
@@ -1074,7 +1140,6 @@ struct Worker {
           op.set_minmax(cur, op.BK(R)[0], op.BK(R)[K - 1]);
           if (first) {
             st_relaxed(&H.meta[cur].state, ST_AVAIL);
-            __threadfence();
             st_release(A.ret + cur, seq);  // return the lent node to the server
           } else {
             release(cur, cur_ticket);
@@ -1115,7 +1180,6 @@ struct Worker {
         op.set_minmax(cur, op.BK(C2)[0], op.BK(C2)[K - 1]);
         if (first) {
           st_relaxed(&H.meta[cur].state, ST_AVAIL);
-          __threadfence();
           st_release(A.ret + cur, seq);
         } else {
           release(cur, cur_ticket);
@@ -1129,10 +1193,12 @@ struct Worker {
 
   __device__ void run() {
     const int tid = threadIdx.x;
+    for (int i = 0; i < 8; ++i) tm[i] = 0;
     for (;;) {
       if (tid == 0) {
         u32 kind = 0, arg = 0;
         u32 ns = 32;
+        const ull ti = clock64();
         for (;;) {
           // body tasks first (they unblock the server)
           const u32 tail = ld_acquire(A.ctl + C_TASK_TAIL);
@@ -1144,6 +1210,7 @@ struct Worker {
             head = prev;
           }
           if (got) {
+            if (C.prog) C.prog[17 + 2 * blockIdx.x] = 0xD0000000u | head;
             while (ld_acquire(A.task_pub + (head % NTASK)) != head + 1) {}
             kind = ld_relaxed(A.task + (size_t)(head % NTASK) * 8);
             arg = head;
@@ -1165,26 +1232,37 @@ struct Worker {
               break;
             }
           }
+          if (C.prog) {
+            C.prog[17 + 2 * blockIdx.x] = 0xE0000000u | ((ld_relaxed(A.ctl + C_TASK_HEAD) & 0x3FFF) << 14) |
+                                          (ld_relaxed(A.ctl + C_TASK_TAIL) & 0x3FFF);
+            C.prog[16 + 2 * blockIdx.x] = 0xEE000000u | (ld_relaxed(A.ctl + C_DONE) << 16) |
+                                          (ld_relaxed(A.ctl + C_SORT_NEXT) & 0xFFFF);
+          }
           if (ld_acquire(A.ctl + C_DONE) && ld_relaxed(A.ctl + C_TASK_HEAD) >= ld_acquire(A.ctl + C_TASK_TAIL)) {
             kind = 0xFFFFFFFFu;
             break;
           }
           __nanosleep(ns);
-          ns = ns < 256 ? ns * 2 : 256;
+          ns = ns < 1024 ? ns * 2 : 1024;
         }
         op.ctl->b[8] = kind; op.ctl->b[9] = arg;
+        tm[3] += clock64() - ti;
       }
       cta_bar<NT>();
       const u32 kind = op.ctl->b[8], arg = op.ctl->b[9];
       cta_bar<NT>();
       if (kind == 0xFFFFFFFFu) break;
-      if (kind == 3) sort_job(arg);
-      else if (kind == TASK_INS) ins_body(arg);
-      else if (kind == TASK_DEL) del_body(arg);
+      const ull tw = clock64();
+      if (tid == 0 && C.prog) { C.prog[16 + 2 * blockIdx.x] = (kind << 24) | (arg & 0xFFFFFF); C.prog[17 + 2 * blockIdx.x] = 0; }
+      if (kind == 3) { sort_job(arg); if (tid == 0) { tm[0] += clock64() - tw; tm[6]++; } }
+      else if (kind == TASK_INS) { ins_body(arg); if (tid == 0) { tm[1] += clock64() - tw; tm[4]++; } }
+      else if (kind == TASK_DEL) { del_body(arg); if (tid == 0) { tm[2] += clock64() - tw; tm[5]++; } }
     }
     if (tid == 0) {
       ull* stat = reinterpret_cast<ull*>(H.hdr + H_STAT);
       for (int i = 0; i < NSTAT; ++i) if (op.st[i]) atomicAdd(stat + i, op.st[i]);
+      ull* tms = reinterpret_cast<ull*>(H.hdr + H_TIME) + 16;
+      for (int i = 0; i < 8; ++i) if (tm[i]) atomicAdd(tms + i, tm[i]);
     }
   }
 };

@@ -13,12 +13,13 @@ __global__ void k_merge(const u32* in, long long* out, int reps) {
   long long t0 = clock64();
   for (int r = 0; r < reps; ++r) {
     if (MODE == 0) cta_merge_split<NT, false>(z, nullptr, K, w, nullptr, K, K, x, nullptr, y, nullptr);
-    else cta_rank_merge<K, NT, false>(z, nullptr, K, w, nullptr, K, K, x, nullptr, y, nullptr);
+    else if (MODE == 1) cta_rank_merge<K, NT, false>(z, nullptr, K, w, nullptr, K, K, x, nullptr, y, nullptr);
+    else cta_path_merge<K, NT, false>(z, nullptr, K, w, nullptr, K, K, x, nullptr, y, nullptr);
     __syncthreads();
   }
   long long t1 = clock64();
   if (threadIdx.x == 0) out[0] = (t1 - t0) / reps;
-  if (threadIdx.x == 0) out[1] = x[5] + y[7];
+  if (threadIdx.x == 0) { long long h = 0; for (int i = 0; i < K; ++i) h = h * 31 + x[i] * 7 + y[i]; out[1] = h; }
 }
 
 template <int NT, int K>
@@ -114,8 +115,8 @@ int main() {
   for (int i = 0; i < K; ++i) { a += hin[i] >> 22; b += hin[K + i] >> 22; zz[2 * i] = a; zz[2 * i + 1] = b; }
   cudaMemcpy(d, zz, 8 * K, cudaMemcpyHostToDevice);
 #define MB(NT_, M_) k_merge<NT_, K, M_><<<1, NT_>>>(d, o, 100); cudaMemcpy(h, o, 16, cudaMemcpyDeviceToHost); \
-  printf("%s 2x%d NT=%d: %lld cycles\n", M_ ? "rank_merge" : "merge_path", K, NT_, h[0]);
-  MB(512, 0) MB(1024, 0) MB(256, 0) MB(512, 1) MB(1024, 1) MB(256, 1) MB(128, 1)
+  printf("hash %lld  ", h[1]); printf("%s 2x%d NT=%d: %lld cycles\n", M_ == 2 ? "path_merge_v2" : M_ ? "rank_merge" : "merge_path", K, NT_, h[0]);
+  MB(512, 0) MB(512, 1) MB(1024, 1) MB(512, 2) MB(1024, 2) MB(256, 2)
   cudaMemcpy(d, hin, 16 * K, cudaMemcpyHostToDevice);
   k_sort<512, K><<<1, 512>>>(d, o, 50); cudaMemcpy(h, o, 16, cudaMemcpyDeviceToHost);
   printf("cta_sort %d NT=512: %lld cycles\n", K, h[0]);
