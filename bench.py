@@ -150,7 +150,7 @@ def _config(args):
                          f"then deletemin all, K={args.K}, {'key+value' if args.values else 'keys only'} "
                          f"(w={w} B)"),
             "n_keys": 1 << args.n_log2, "K": args.K, "w_bytes": w, "dist": args.dist,
-            "threads_per_cta": 512, "l2": f"inputs and heap ({(1 << args.n_log2) * w * 3 >> 20} MiB) "
+            "threads_per_cta": 512, "execution": args.mode, "l2": f"inputs and heap ({(1 << args.n_log2) * w * 3 >> 20} MiB) "
                                           "larger than the 126 MB L2; no flush"}
 
 
@@ -188,6 +188,8 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--profile-steps", type=int, default=0, help="ncu mode: run N untimed steps and exit")
+    ap.add_argument("--mode", default="locks", choices=["locks", "server"],
+                    help="execution: paper-literal per-node locks on all CTAs, or root-server CTA")
     args = ap.parse_args()
     world, rank, local = _dist_setup()
 
@@ -212,7 +214,7 @@ def main():
     dv = torch.arange(n, dtype=torch.int32, device="cuda") if args.values else None
     out_k = torch.empty(n, dtype=torch.int32, device="cuda")
     out_v = torch.empty(n, dtype=torch.int32, device="cuda") if args.values else None
-    q = pkg.BGPQ(capacity=n, K=K, values=args.values)
+    q = pkg.BGPQ(capacity=n, K=K, values=args.values, locks=(args.mode == "locks"))
     stream = torch.cuda.current_stream()
 
     def step(ev=None):
