@@ -103,6 +103,21 @@ def byte_model(st: dict, K: int, w: int) -> dict:
     return {"insert": ins, "deletemin": dele, "total": ins + dele, "insert_noop_skipped": skipped}
 
 
+def max_over_ranks(ms: float, dist=None, device: str = "cpu") -> float:
+    """Max of a per-rank time over all ranks (replicas: the job ends with its slowest GPU)."""
+    if dist is None:
+        return ms
+    import torch
+    t = torch.tensor([float(ms)], dtype=torch.float64, device=device)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
+def job_throughput(n_keys: int, steps: int, world: int, total_ms: float) -> float:
+    """Whole-job keys/s: every rank processes n_keys per step (weak scaling, replicas)."""
+    return world * n_keys * steps / (total_ms / 1e3)
+
+
 def _dist_setup():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -260,12 +275,9 @@ def main():
     total_ms = t_start.elapsed_time(t_end)
     ins_ms = [e[0].elapsed_time(e[1]) for e in evs]
     del_ms = [e[1].elapsed_time(e[2]) for e in evs]
-    if dist:
-        t = torch.tensor([total_ms], device="cuda")
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        total_ms = float(t.item())
+    total_ms = max_over_ranks(total_ms, dist, device="cuda")
     ms_per_step = total_ms / args.steps
-    value = world * n * args.steps / (total_ms / 1e3)
+    value = job_throughput(n, args.steps, world, total_ms)
 
     dst = {k: (st1[k] - st0[k]) // args.steps for k in st1}
     bm = byte_model(dst, K, w)
