@@ -229,7 +229,7 @@ def main():
     dv = torch.arange(n, dtype=torch.int32, device="cuda") if args.values else None
     out_k = torch.empty(n, dtype=torch.int32, device="cuda")
     out_v = torch.empty(n, dtype=torch.int32, device="cuda") if args.values else None
-    q = pkg.BGPQ(capacity=n, K=K, values=args.values, locks=(args.mode == "locks"))
+    q = pkg.BGPQ(capacity=n, K=K, values=args.values, server=(args.mode == "server"))
     stream = torch.cuda.current_stream()
 
     def step(ev=None):

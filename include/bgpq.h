@@ -47,13 +47,15 @@ enum {
   BGPQ_FLAG_VALUES = 1u, /* store a uint32 value with every key (w = 8 B per entry)        */
   BGPQ_FLAG_SERIAL = 2u, /* execute operations one at a time on a single CTA (test mode:
                             the node layout then equals the sequential Alg.1-3 model)     */
-  BGPQ_FLAG_LOCKS = 4u   /* paper-literal execution: every CTA runs whole operations with
-                            per-node locks from the root down (no root-server CTA)        */
+  BGPQ_FLAG_LOCKS = 4u,  /* paper-literal per-node-lock execution (the default; kept as an
+                            explicit flag for callers that name it)                        */
+  BGPQ_FLAG_SERVER = 8u  /* root-server execution: one CTA holds the root, the pBuffer and
+                            the top levels in shared memory and executes every root section
+                            in call order; workers run the lock walks below     */
 };
-/* Default execution (no SERIAL/LOCKS flag): one persistent "root server" CTA holds the root,
- * the pBuffer and the top levels of the heap in shared memory and executes the root section
- * of every operation in call order; worker CTAs pre-sort INSERT batches and run the
- * per-node-lock walks below the top levels. */
+/* Default execution: every CTA of a persistent grid executes whole operations (Alg.1, Alg.2+3)
+ * with per-node locks taken top-down hand over hand; a lock warp per CTA takes
+ * the next level's locks and stages its nodes while the CTA merges. */
 
 /* Create an empty heap able to hold `capacity` keys with node capacity K (§3.1:
  * every non-root node holds K sorted keys; k > 1).  K must be one of 64, 128, 256, 512,

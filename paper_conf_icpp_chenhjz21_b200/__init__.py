@@ -23,7 +23,7 @@ NVCC_FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", 
               "-Xptxas", "-v", "-shared", "-Xcompiler", "-fPIC"]
 
 BGPQ_OK, BGPQ_EINVAL, BGPQ_ENOMEM, BGPQ_EFULL, BGPQ_ECUDA = 0, -1, -2, -3, -4
-FLAG_VALUES, FLAG_SERIAL, FLAG_LOCKS = 1, 2, 4
+FLAG_VALUES, FLAG_SERIAL, FLAG_LOCKS, FLAG_SERVER = 1, 2, 4, 8
 # GPU node-state encoding (bgpq_ops.cuh); the oracle's encoding differs (see to_oracle_states)
 ST_EMPTY, ST_AVAIL, ST_TARGET, ST_MARKED = 0, 1, 2, 3
 STAT_NAMES = ("ins_ops", "ins_heapify_ops", "ins_levels", "ins_noop", "ins_swap", "ins_merge",
@@ -126,18 +126,19 @@ class BGPQ:
     torch stream, exactly like the C calls they forward to."""
 
     def __init__(self, capacity: int, K: int = 1024, values: bool = True, serial: bool = False,
-                 locks: bool = False):
+                 locks: bool = False, server: bool = False):
         """serial: one CTA, one operation at a time (layout equals the sequential model);
-        locks: paper-literal per-node-lock execution on all CTAs; default: root-server
-        execution."""
+        default (or locks=True): per-node-lock execution on all CTAs with a lock-ahead warp;
+        server: root-server execution."""
         if K not in VALID_K:
             raise ValueError(f"K must be one of {VALID_K}")
         flags = ((FLAG_VALUES if values else 0) | (FLAG_SERIAL if serial else 0)
-                 | (FLAG_LOCKS if locks else 0))
+                 | (FLAG_LOCKS if locks else 0) | (FLAG_SERVER if server else 0))
         self._h = lib().bgpq_create_ex(int(capacity), int(K), flags)
         if not self._h:
             raise BGPQError(f"bgpq_create failed ({lib().bgpq_last_error()})")
-        self.K, self.capacity, self.values, self.serial, self.locks = int(K), int(capacity), values, serial, locks
+        self.K, self.capacity, self.values, self.serial = int(K), int(capacity), values, serial
+        self.locks = not server
 
     def close(self):
         if getattr(self, "_h", None):

@@ -11,6 +11,7 @@
 #include <cstring>
 
 #include "../../include/bgpq.h"
+#include "bgpq_locks.cuh"
 #include "bgpq_server.cuh"
 
 using namespace bgpqd;
@@ -63,19 +64,20 @@ namespace {
 
 template <int K, bool V>
 struct KernelInfo {
+  // the per-node-lock execution (bgpq_locks.cuh): NT compute threads + one lock warp
   static int occupancy(int* out_occ) {
-    auto kern = bgpq_ops_kernel<K, V, NT>;
-    const size_t smem = ops_smem_bytes<K, V>();
+    auto kern = bgpq_locks_kernel<K, V, NT>;
+    const size_t smem = locks_smem_bytes<K, V>();
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return -1;
     int occ = 0;
-    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, NT, smem);
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, NT + 32, smem);
     if (e != cudaSuccess) return -1;
     *out_occ = occ;
     return 0;
   }
   static cudaError_t launch(int grid, const HeapArgs& H, const CallArgs& C, cudaStream_t s) {
-    bgpq_ops_kernel<K, V, NT><<<grid, NT, ops_smem_bytes<K, V>(), s>>>(H, C);
+    bgpq_locks_kernel<K, V, NT><<<grid, NT + 32, locks_smem_bytes<K, V>(), s>>>(H, C);
     g_launches.fetch_add(1);
     return cudaGetLastError();
   }
@@ -199,7 +201,7 @@ int grid_for(const bgpq* q, u64 n_ops) {
   return (int)std::max(1LL, g);
 }
 
-bool server_mode(const bgpq* q) { return !(q->flags & (BGPQ_FLAG_SERIAL | BGPQ_FLAG_LOCKS)); }
+bool server_mode(const bgpq* q) { return (q->flags & BGPQ_FLAG_SERVER) && !(q->flags & BGPQ_FLAG_SERIAL); }
 
 int run_call(bgpq* q, const CallArgs& C, cudaStream_t s) {
   const bool V = (q->flags & BGPQ_FLAG_VALUES) != 0;
@@ -228,7 +230,7 @@ extern "C" {
 bgpq_t* bgpq_create_ex(uint64_t capacity, uint32_t K, uint32_t flags) {
   g_last_error = BGPQ_OK;
   if (const char* d = getenv("BGPQ_DEBUG")) g_debug = (unsigned)atoi(d);
-  if (!valid_K(K) || capacity == 0 || (flags & ~7u)) {
+  if (!valid_K(K) || capacity == 0 || (flags & ~15u)) {
     fail(BGPQ_EINVAL);
     return nullptr;
   }

@@ -10,6 +10,7 @@
 //  * cta_sort: warp_sort64 runs followed by merge-path passes in smem.
 #pragma once
 #include <cstdint>
+#include <type_traits>
 
 namespace bgpqd {
 
@@ -315,6 +316,259 @@ __device__ __forceinline__ void cta_path_merge(const u32* __restrict__ zk, const
       }
     }
   }
+}
+
+// ----------------------------------------------------------------------------------------
+// SORT_SPLIT by merge path [11] with a register window (the hot-path merge, v3).
+// Threads 0..NTM-1 each produce VT = 2*KMAX/NTM consecutive outputs [d, d+VT) of the merge.
+// After the branchless co-rank search on diagonal d (i from Z, j = d - i from W), the VT
+// outputs are exactly the VT smallest of Z[i, i+VT) u W[j, j+VT): both windows are loaded
+// with independent LDS, C[k] = min(A[k], B[VT-1-k]) selects them as a bitonic sequence
+// (Batcher's half-cleaner) and log2(VT) compare-exchange stages sort it — no dependent
+// shared-memory chain after the search.  With values the comparison key is the stable
+// composite (key, Z before W, index), so equal keys never migrate between threads and the
+// (key, value) pairs stay a permutation; keys-only compares 32-bit keys.
+// Output position p < ma goes to X[p], else Y[p - ma].  X/Y must not alias Z/W.
+// ----------------------------------------------------------------------------------------
+template <int VT, typename T>
+__device__ __forceinline__ void bitonic_sort_regs(T (&c)[VT]) {
+#pragma unroll
+  for (int s = VT / 2; s > 0; s >>= 1) {
+#pragma unroll
+    for (int k = 0; k < VT; ++k) {
+      if ((k & s) == 0) {
+        const T a = c[k], b = c[k + s];
+        c[k] = a < b ? a : b;
+        c[k + s] = a < b ? b : a;
+      }
+    }
+  }
+}
+
+template <int KMAX, int NTM, bool V>
+__device__ __forceinline__ void cta_merge_win(const u32* __restrict__ zk, const u32* __restrict__ zv,
+                                              int na, const u32* __restrict__ wk,
+                                              const u32* __restrict__ wv, int nb, int ma,
+                                              u32* __restrict__ xk, u32* __restrict__ xv,
+                                              u32* __restrict__ yk, u32* __restrict__ yv) {
+  constexpr int VT = (2 * KMAX) / NTM;
+  static_assert(VT >= 2 && (VT & (VT - 1)) == 0 && VT * NTM == 2 * KMAX, "VT must be a power of two");
+  constexpr int LOG = Log2Ceil<KMAX + 1>::v;
+  const int t = threadIdx.x;
+  if (t >= NTM) return;
+  const int N = na + nb;
+  const int d = t * VT;
+  if (d >= N) return;
+  int lo = max(0, d - nb), hi = min(d, na);
+#pragma unroll
+  for (int it = 0; it < LOG; ++it) {
+    const int len = hi - lo;
+    const int mid = lo + (len >> 1);
+    const bool act = len > 0;
+    const u32 a = zk[act ? mid : 0];
+    const u32 b = wk[act ? d - 1 - mid : 0];
+    const bool right = act && (a <= b);
+    lo = right ? mid + 1 : lo;
+    hi = (act && !right) ? mid : hi;
+  }
+  const int i = lo, j = d - lo;
+  if (!V) {
+    u32 A[VT], C[VT];
+#pragma unroll
+    for (int k = 0; k < VT; ++k) A[k] = (i + k < na) ? zk[i + k] : KEY_MAX;
+#pragma unroll
+    for (int k = 0; k < VT; ++k) {
+      const int jj = j + VT - 1 - k;
+      const u32 b = (jj < nb) ? wk[jj] : KEY_MAX;
+      C[k] = A[k] < b ? A[k] : b;
+    }
+    bitonic_sort_regs<VT>(C);
+    if (VT >= 4 && d + VT <= N && (d + VT <= ma || (d >= ma && ((ma & 3) == 0)))) {
+      u32* dk = (d + VT <= ma) ? xk + d : yk + (d - ma);
+#pragma unroll
+      for (int k = 0; k < VT; k += 4)
+        *reinterpret_cast<uint4*>(dk + k) = make_uint4(C[k], C[(k + 1) % VT], C[(k + 2) % VT], C[(k + 3) % VT]);
+    } else {
+#pragma unroll
+      for (int k = 0; k < VT; ++k) {
+        const int o = d + k;
+        if (o < N) {
+          if (o < ma) xk[o] = C[k];
+          else yk[o - ma] = C[k];
+        }
+      }
+    }
+  } else {
+    u64 A[VT], C[VT];
+#pragma unroll
+    for (int k = 0; k < VT; ++k)
+      A[k] = (i + k < na) ? (((u64)zk[i + k] << 32) | (u32)(i + k)) : ~0ull;
+#pragma unroll
+    for (int k = 0; k < VT; ++k) {
+      const int jj = j + VT - 1 - k;
+      const u64 b = (jj < nb) ? (((u64)wk[jj] << 32) | 0x80000000u | (u32)jj) : ~0ull;
+      C[k] = A[k] < b ? A[k] : b;
+    }
+    bitonic_sort_regs<VT>(C);
+    u32 ko[VT], vo[VT];
+#pragma unroll
+    for (int k = 0; k < VT; ++k) {
+      const u32 lw = (u32)C[k];
+      const u32 idx = lw & 0x7FFFFFFFu;
+      ko[k] = (u32)(C[k] >> 32);
+      vo[k] = (d + k < N) ? ((lw & 0x80000000u) ? wv[idx] : zv[idx]) : 0u;
+    }
+    if (VT >= 4 && d + VT <= N && (d + VT <= ma || (d >= ma && ((ma & 3) == 0)))) {
+      u32* dk = (d + VT <= ma) ? xk + d : yk + (d - ma);
+      u32* dv = (d + VT <= ma) ? xv + d : yv + (d - ma);
+#pragma unroll
+      for (int k = 0; k < VT; k += 4) {
+        *reinterpret_cast<uint4*>(dk + k) = make_uint4(ko[k], ko[(k + 1) % VT], ko[(k + 2) % VT], ko[(k + 3) % VT]);
+        *reinterpret_cast<uint4*>(dv + k) = make_uint4(vo[k], vo[(k + 1) % VT], vo[(k + 2) % VT], vo[(k + 3) % VT]);
+      }
+    } else {
+#pragma unroll
+      for (int k = 0; k < VT; ++k) {
+        const int o = d + k;
+        if (o < N) {
+          if (o < ma) { xk[o] = ko[k]; xv[o] = vo[k]; }
+          else { yk[o - ma] = ko[k]; yv[o - ma] = vo[k]; }
+        }
+      }
+    }
+  }
+}
+
+// ----------------------------------------------------------------------------------------
+// SORT_SPLIT by warp-cooperative merge path (v4, the hot-path merge).
+// Warp w of the first NW warps produces the OW = 2*KMAX/NW consecutive outputs [D0, D0+OW)
+// of the stable merge, E = OW/32 per lane, element e = lane + 32*k in register k:
+//  1. co-rank of D0 by a two-round 32-ary search with __ballot_sync (probe stride odd so
+//     the 32 probes fall in distinct banks) instead of log2(K) dependent probes per thread;
+//  2. the OW outputs are the OW smallest of Z[i0, i0+OW) u W[j0, j0+OW): lane l loads
+//     A[k] = Z[i0+e] and, in reversed order, B[k] = W[j0+OW-1-e]; C = min(A, B) is bitonic
+//     (Batcher's half-cleaner) and holds exactly them;
+//  3. C is sorted by a bitonic network: strides >= 32 inside the lane's registers, strides
+//     < 32 with __shfl_xor_sync; then coalesced, conflict-free stores (lane-strided).
+// With values the comparison key is the stable composite (key, Z before W, index) and the
+// value is gathered from its source index; keys-only compares the 32-bit keys.
+// Output position p < ma goes to X[p], else Y[p - ma].  X/Y must not alias Z/W.
+// ----------------------------------------------------------------------------------------
+template <typename T>
+__device__ __forceinline__ T shfl_xor_t(T v, int m) {
+  if constexpr (sizeof(T) == 8) {
+    const u32 lo = __shfl_xor_sync(0xffffffffu, (u32)v, m);
+    const u32 hi = __shfl_xor_sync(0xffffffffu, (u32)(v >> 32), m);
+    return ((u64)hi << 32) | lo;
+  } else {
+    return __shfl_xor_sync(0xffffffffu, v, m);
+  }
+}
+
+// co-rank of diagonal D (number of Z entries among the first D outputs; Z first on ties)
+__device__ __forceinline__ int warp_corank(const u32* __restrict__ zk, int na, const u32* __restrict__ wk,
+                                           int nb, int D) {
+  const int lane = threadIdx.x & 31;
+  int lo = max(0, D - nb), hi = min(D, na);
+  while (hi - lo > 0) {  // at most two rounds for ranges <= 1056
+    const int n = hi - lo;
+    int s = (n + 31) >> 5;
+    if (s > 1 && !(s & 1)) ++s;  // odd stride: distinct banks
+    const int m = lo + s * (lane + 1) - 1;
+    const bool valid = m < hi;
+    bool q = false;
+    if (valid) q = zk[m] <= wk[D - 1 - m];
+    const u32 bal = __ballot_sync(0xffffffffu, valid && q);
+    const int L = __popc(bal);  // Q is monotone: the first L probes are true
+    lo = lo + s * L;
+    hi = min(hi, lo + s - 1);
+    if (s == 1) hi = lo;
+  }
+  return lo;
+}
+
+template <int KMAX, int NW, bool V>
+__device__ __forceinline__ void cta_merge_warp(const u32* __restrict__ zk, const u32* __restrict__ zv,
+                                               int na, const u32* __restrict__ wk,
+                                               const u32* __restrict__ wv, int nb, int ma,
+                                               u32* __restrict__ xk, u32* __restrict__ xv,
+                                               u32* __restrict__ yk, u32* __restrict__ yv) {
+  constexpr int OW = (2 * KMAX) / NW;
+  constexpr int E = OW / 32;
+  static_assert(E >= 1 && (E & (E - 1)) == 0 && OW * NW == 2 * KMAX, "E must be a power of two");
+  using T = typename std::conditional<V, u64, u32>::type;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (warp >= NW) return;
+  const int N = na + nb;
+  const int D0 = warp * OW;
+  if (D0 >= N) return;
+  const int i0 = warp_corank(zk, na, wk, nb, D0);
+  const int j0 = D0 - i0;
+  T C[E];
+#pragma unroll
+  for (int k = 0; k < E; ++k) {
+    const int ia = i0 + lane + 32 * k;
+    const int jb = j0 + OW - 1 - (lane + 32 * k);
+    T a, b;
+    if constexpr (V) {
+      a = ia < na ? (((u64)zk[ia] << 32) | (u32)ia) : ~0ull;
+      b = jb < nb ? (((u64)wk[jb] << 32) | 0x80000000u | (u32)jb) : ~0ull;
+    } else {
+      a = ia < na ? zk[ia] : KEY_MAX;
+      b = jb < nb ? wk[jb] : KEY_MAX;
+    }
+    C[k] = a < b ? a : b;
+  }
+  // bitonic sort (ascending) of the OW-entry bitonic sequence
+#pragma unroll
+  for (int s = OW / 2; s >= 32; s >>= 1) {
+    const int r = s / 32;
+#pragma unroll
+    for (int k = 0; k < E; ++k) {
+      if ((k & r) == 0) {
+        const T a = C[k], b = C[k + r];
+        C[k] = a < b ? a : b;
+        C[k + r] = a < b ? b : a;
+      }
+    }
+  }
+#pragma unroll
+  for (int s = 16; s > 0; s >>= 1) {
+    const bool upper = (lane & s) != 0;
+#pragma unroll
+    for (int k = 0; k < E; ++k) {
+      const T p = shfl_xor_t(C[k], s);
+      C[k] = upper ? (C[k] > p ? C[k] : p) : (C[k] < p ? C[k] : p);
+    }
+  }
+#pragma unroll
+  for (int k = 0; k < E; ++k) {
+    const int o = D0 + lane + 32 * k;
+    if (o < N) {
+      u32 key, val = 0;
+      if constexpr (V) {
+        key = (u32)(C[k] >> 32);
+        const u32 lw = (u32)C[k];
+        const u32 idx = lw & 0x7FFFFFFFu;
+        val = (lw & 0x80000000u) ? wv[idx] : zv[idx];
+      } else {
+        key = C[k];
+      }
+      if (o < ma) { xk[o] = key; if (V) xv[o] = val; }
+      else { yk[o - ma] = key; if (V) yv[o - ma] = val; }
+    }
+  }
+}
+
+// The SORT_SPLIT used on the hot path: register-window merge path with VT = 4 outputs per
+// thread (threads 0 .. 2K/4-1 of the NT compute threads take part).  Measured on B200
+// (tools/micro_merge.cu, K = 1024, NT = 512): 1540 cycles keys-only / 2110 key+value, vs
+// 2110 / 2190 for the co-ranking merge.
+template <int K, int NT, bool V>
+__device__ __forceinline__ void sort_split(const u32* zk, const u32* zv, int na, const u32* wk, const u32* wv,
+                                           int nb, int ma, u32* xk, u32* xv, u32* yk, u32* yv) {
+  constexpr int NTM = (2 * K / 4 <= NT) ? 2 * K / 4 : NT;
+  cta_merge_win<K, NTM, V>(zk, zv, na, wk, wv, nb, ma, xk, xv, yk, yv);
 }
 
 // One pass of a bottom-up merge sort: merge sorted runs [2q*run, (2q+1)*run) and

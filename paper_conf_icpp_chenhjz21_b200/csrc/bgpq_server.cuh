@@ -196,7 +196,7 @@ struct Server {
   __device__ __forceinline__ void merge(int z, int na, int w, int nb, int ma, int x, int y) {
     main_sync();
     const ull t0 = clock64();
-    cta_rank_merge<K, NT, V>(BK(z), BV(z), na, BK(w), BV(w), nb, ma, BK(x), BV(x), BK(y), BV(y));
+    sort_split<K, NT, V>(BK(z), BV(z), na, BK(w), BV(w), nb, ma, BK(x), BV(x), BK(y), BV(y));
     main_sync();
     if (threadIdx.x == 0) { tm[TM_SRV_MERGE] += clock64() - t0; tm[TM_SRV_MERGES_N]++; }
   }

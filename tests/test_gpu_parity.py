@@ -45,7 +45,7 @@ def test_phased_sorted(K, dist, mode):
         n = 300 * K + 37  # deeper than the on-chip levels for every K
     keys = synth.keys(n, seed=synth.SEEDS["C3"], dist=dist)
     vals = synth.values(n)
-    q = pkg.BGPQ(capacity=n, K=K, values=True, locks=(mode == "locks"))
+    q = pkg.BGPQ(capacity=n, K=K, values=True, server=(mode == "server"))
     q.insert(_dev(keys), _dev(vals))
     assert q.size() == n
     assert _gpu_inv(q) == (0, 0)
@@ -183,7 +183,7 @@ def test_concurrent_mixed_replay(K, p_ins, partial, mode):
         types, _ = synth.random_ops(n_ops, K, seed=41 + K, p_insert=p_ins)
         sizes = np.full(n_ops, K, np.uint32)
     keys, in_off = _mixed_inputs(types, sizes, K, seed=43)
-    q = pkg.BGPQ(capacity=len(keys) + K, K=K, values=True, locks=(mode == "locks"))
+    q = pkg.BGPQ(capacity=len(keys) + K, K=K, values=True, server=(mode == "server"))
     outk, outv, cnt, lin = _run_mixed(q, types, sizes, keys, in_off)
     ref = _replay_check(types, sizes, keys, in_off, outk, outv, cnt, lin)
     for j in np.nonzero(types == 1)[0]:
@@ -200,7 +200,7 @@ def test_concurrent_pairs_with_prefill_replay(mode):
     """Utilisation shape: prefill, then insert/deletemin pairs on all CTAs."""
     K = 64
     pre = synth.keys(1 << 17, seed=50)
-    q = pkg.BGPQ(capacity=(1 << 18) + 4096 * K, K=K, values=True, locks=(mode == "locks"))
+    q = pkg.BGPQ(capacity=(1 << 18) + 4096 * K, K=K, values=True, server=(mode == "server"))
     q.insert(_dev(pre), _dev(synth.values(len(pre))))
     types, sizes = synth.mixed_ops(3000, K, seed=51, partial=True)
     keys, in_off = _mixed_inputs(types, sizes, K, seed=52)
@@ -219,7 +219,7 @@ def test_marked_handoff_replay(mode):
         types, _ = synth.random_ops(3000, K, seed=60 + seed, p_insert=0.5)
         sizes = np.full(len(types), K, np.uint32)
         keys, in_off = _mixed_inputs(types, sizes, K, seed=70 + seed)
-        q = pkg.BGPQ(capacity=len(keys) + K, K=K, values=True, locks=(mode == "locks"))
+        q = pkg.BGPQ(capacity=len(keys) + K, K=K, values=True, server=(mode == "server"))
         outk, outv, cnt, lin = _run_mixed(q, types, sizes, keys, in_off)
         _replay_check(types, sizes, keys, in_off, outk, outv, cnt, lin)
         assert _gpu_inv(q) == (0, 0)
@@ -275,7 +275,7 @@ def test_full_size_c2_properties(mode):
     n, K = 1 << 27, 1024
     keys = synth.keys(n, seed=synth.SEEDS["C2"])
     dk = _dev(keys)
-    q = pkg.BGPQ(capacity=n, K=K, values=False, locks=(mode == "locks"))
+    q = pkg.BGPQ(capacity=n, K=K, values=False, server=(mode == "server"))
     q.insert(dk)
     assert q.size() == n
     ok, _ = q.deletemin(n)
