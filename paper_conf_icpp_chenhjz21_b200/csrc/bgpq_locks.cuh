@@ -25,6 +25,18 @@
 namespace bgpqd {
 
 constexpr int LSLOT = 10;  // smem node slots
+#ifndef BGPQ_T_MARK
+#define BGPQ_T_MARK 1
+#endif
+#ifndef BGPQ_JOINT_RELEASE
+#define BGPQ_JOINT_RELEASE 1
+#endif
+#ifndef BGPQ_PREFETCH
+#define BGPQ_PREFETCH 1
+#endif
+#ifndef BGPQ_HDR_BATCH
+#define BGPQ_HDR_BATCH 1
+#endif
 
 struct LCtl {
   u64 bar;      // compute-thread TMA loads
@@ -39,11 +51,15 @@ struct LCtl {
   u32 p_st[2], p_min[2], p_max[2];
   // agent T mailbox
   u32 t_req;
+  u32 t_kind;  // 0: take the refill node (Alg.2 l.6-12); 1: mark tar TARGET (Alg.1 l.5-6)
   u32 t_node, t_slot, t_rootload, t_rootpar;
   u32 t_marked;
   u32 t_done;
   u32 stop;
+  ull st[NSTAT];  // thread 0's device counters (shared memory: gpu-scope acquires and fences
+  ull tm[32];     // invalidate L1, so local-memory counters would cost an L2 round trip)
 };
+constexpr size_t LCTL_BYTES = (sizeof(LCtl) + 127) / 128 * 128;  // node slots start here
 
 __device__ __forceinline__ u32 ld_acq_cta(const u32* p) {
   u32 v;
@@ -68,7 +84,7 @@ enum : int {
   LT_DEL_TOTAL = 0, LT_DEL_ROOTACQ, LT_DEL_ROOTHOLD, LT_DEL_ROOTLOAD, LT_DEL_TWAIT, LT_DEL_PWAIT,
   LT_DEL_MERGE, LT_DEL_STORE, LT_DEL_LEVELS, LT_INS_TOTAL, LT_INS_SORT, LT_INS_ROOTACQ,
   LT_INS_ROOTHOLD, LT_INS_PWAIT, LT_INS_MERGE, LT_INS_STORE, LT_INS_TARWAIT, LT_P_LOCKWAIT,
-  LT_T_LOCKWAIT, LT_T_TOTAL, LT_N
+  LT_T_LOCKWAIT, LT_T_TOTAL, LT_R1, LT_R2, LT_R3, LT_R4, LT_R5, LT_R6, LT_R7, LT_N
 };
 
 template <int K, bool V, int NT>
@@ -76,18 +92,22 @@ struct OpL {
   static constexpr u32 NBYTES = K * 4u;
   HeapArgs H;
   bool timing;
-  ull tm[LT_N];
+  ull* tm;  // -> ctl->tm
   int tmerge = LT_DEL_MERGE, tstore = LT_DEL_STORE;  // timer ids of the current op type
   __device__ __forceinline__ ull now() const { return timing ? clock64() : 0ull; }
   __device__ __forceinline__ void acc(int id, ull t0) { if (timing && threadIdx.x == 0) tm[id] += clock64() - t0; }
+  ull tmark;  // root-hold section marks (thread 0)
+  __device__ __forceinline__ void mark(int id) {
+    if (timing && threadIdx.x == 0) { const ull t = clock64(); tm[id] += t - tmark; tmark = t; }
+  }
   u32* sk;
   u32* sv;
   LCtl* ctl;
   u32 mphase;      // ctl->bar phase (all compute threads)
-  u32 pphase[2];   // pbar phases (all compute threads)
+  u32 pph;         // pbar[0] / pbar[1] phases in bits 0 / 1 (registers, not a local array)
   u32 tphase;      // tbar phase (all compute threads)
   u32 pb;          // next pbar index
-  ull st[NSTAT];   // thread 0's counters
+  ull* st;         // -> ctl->st (thread 0's counters)
 
   __device__ __forceinline__ u32* BK(int s) const { return sk + s * K; }
   __device__ __forceinline__ u32* BV(int s) const { return V ? sv + s * K : nullptr; }
@@ -156,6 +176,39 @@ struct OpL {
       if (V && ov) ov[pos + i] = BV(s)[off + i];
     }
   }
+  // One round trip for the words the root lock protects: {heapSize, |root|, |pBuffer|, err},
+  // the per-call ticket, the 64-bit linearization ticket, min(pBuffer) and max(root).
+  struct Hdr { u32 hs, rs, ps, call, pbmin, rootmax; ull lin; };
+  __device__ __forceinline__ Hdr hdr_load() const {
+    Hdr h;
+#if !BGPQ_HDR_BATCH
+    h.lin = lin_get(); h.call = hget(H_CALL); h.hs = hget(H_HS); h.rs = hget(H_RS); h.ps = hget(H_PS);
+    h.pbmin = ld_relaxed(&H.meta[0].kmin); h.rootmax = ld_relaxed(&H.meta[1].kmax);
+    return h;
+#endif
+    u32 err;
+    asm volatile(
+        "ld.relaxed.gpu.global.v4.u32 {%0, %1, %2, %3}, [%7];\n\t"
+        "ld.relaxed.gpu.global.u32 %4, [%8];\n\t"
+        "ld.relaxed.gpu.global.u64 %5, [%9];\n\t"
+        "ld.relaxed.gpu.global.u32 %6, [%10];"
+        : "=r"(h.hs), "=r"(h.rs), "=r"(h.ps), "=r"(err), "=r"(h.call), "=l"(h.lin), "=r"(h.pbmin)
+        : "l"(H.hdr), "l"(H.hdr + H_CALL), "l"(H.hdr + H_LIN), "l"(&H.meta[0].kmin)
+        : "memory");
+    h.rootmax = ld_relaxed(&H.meta[1].kmax);
+    return h;
+  }
+  // release several node locks behind one gpu-scope fence (the caller's CTA barrier has
+  // ordered every thread's node writes before this thread)
+  __device__ __forceinline__ void release_locks(u32 a, u32 b = 0) const {
+    asm volatile("fence.acq_rel.gpu;" ::: "memory");
+    if (a) st_relaxed(lk(a), 0u);
+    if (b) st_relaxed(lk(b), 0u);
+  }
+  __device__ __forceinline__ void prefetch_l2(u32 node) const {
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(H.gk + (size_t)node * K), "r"(NBYTES) : "memory");
+    if (V) asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(H.gv + (size_t)node * K), "r"(NBYTES) : "memory");
+  }
   __device__ __forceinline__ ull lin_get() const {
     ull v;
     asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(H.hdr + H_LIN) : "memory");
@@ -175,12 +228,20 @@ struct OpL {
   // compute threads: wait for the P request issued on pbar[pb]; advances pb
   __device__ __forceinline__ void wait_p(int id) {
     const ull t0 = now();
-    mbar_wait(&ctl->pbar[pb], pphase[pb]);
+    mbar_wait(&ctl->pbar[pb], (pph >> pb) & 1u);
     acc(id, t0);
-    pphase[pb] ^= 1u;
+    pph ^= 1u << pb;
     pb ^= 1u;
   }
+  __device__ __forceinline__ void post_mark(u32 tar) {
+    ctl->t_kind = 1u; ctl->t_node = tar;
+    st_rel_cta(&ctl->t_req, ctl->t_req + 1u);
+  }
+  __device__ __forceinline__ void wait_t_done() const {
+    while (ld_acq_cta(&ctl->t_done) != ctl->t_req) {}
+  }
   __device__ __forceinline__ void post_t(u32 tar, int slot, u32 rootload) {
+    ctl->t_kind = 0u;
     ctl->t_node = tar; ctl->t_slot = (u32)slot; ctl->t_rootload = rootload; ctl->t_rootpar = mphase;
     st_rel_cta(&ctl->t_req, ctl->t_req + 1u);
   }
@@ -188,10 +249,11 @@ struct OpL {
   // =====================================================================================
   // BGPQ_INSERT (Alg.1).  Keys ik[0:size), values iv (nullable), 1 <= size <= K.
   // =====================================================================================
-  __device__ void insert(const u32* ik, const u32* iv, u32 size, ull* lin_out) {
+  __device__ __forceinline__ void insert(const u32* ik, const u32* iv, u32 size, ull* lin_out) {
     const int tid = threadIdx.x;
     tmerge = LT_INS_MERGE; tstore = LT_INS_STORE;
     const ull t_ins = now();
+    tmark = t_ins;
     cta_bar<NT>();
     if (tid == 0) {
       ctl->b[0] = alloc();
@@ -217,13 +279,13 @@ struct OpL {
       acc(LT_INS_ROOTACQ, ta);
       t_root = now();
       fence_proxy_async();
-      const ull lin = lin_get();
-      lin_set(lin + 1);
-      if (lin_out) *lin_out = lin;
-      ctl->b[0] = hget(H_HS);
-      ctl->b[1] = hget(H_RS);
-      ctl->b[2] = hget(H_PS);
-      ctl->b[3] = ld_relaxed(&H.meta[1].kmax);
+      const Hdr h = hdr_load();
+      lin_set(h.lin + 1);
+      if (lin_out) *lin_out = h.lin;
+      ctl->b[0] = h.hs;
+      ctl->b[1] = h.rs;
+      ctl->b[2] = h.ps;
+      ctl->b[3] = h.rootmax;
     }
     cta_bar<NT>();
     const u32 hs = ctl->b[0], rs = ctl->b[1], ps = ctl->b[2], rootmax = ctl->b[3];
@@ -314,10 +376,15 @@ struct OpL {
       st[S_INS_HEAPIFY]++;
       hset(H_PS, nps);
       hset(H_HS, tar);
-      // l.5-6: LOCK(tar); Heap[tar].state <- TARGET; UNLOCK(tar)
+      // l.5-6: LOCK(tar); Heap[tar].state <- TARGET; UNLOCK(tar) — by agent T; the root is
+      // not released before it is done
+#if BGPQ_T_MARK
+      post_mark(tar);
+#else
       lock_acquire(lk(tar));
       st_relaxed(stp(tar), ST_TARGET);
       lock_release(lk(tar));
+#endif
       if (c != tar) {  // lock-ahead of the first path node (still holding the root)
         const int s = alloc();
         ctl->b[7] = (u32)s;
@@ -339,6 +406,7 @@ struct OpL {
           lock_release(lk(c));  // as if the loop had exited before LOCK(cur)
           free_slot(sc);
         } else {
+          if (held == 1) wait_t_done();
           lock_release(lk(held));  // l.32: UNLOCK(PARENT(cur)) — cur is held
           if (held == 1) acc(LT_INS_ROOTHOLD, t_root);
           dec = (cmax <= imin) ? 0u : (imax <= cmin) ? 1u : 2u;  // l.33 fast paths
@@ -386,6 +454,7 @@ struct OpL {
     cta_bar<NT>();
     if (tid == 0) {
       const ull tt = now();
+      if (held == 1) wait_t_done();  // agent T's LOCK(tar) of l.5-6 must be over first
       lock_acquire(lk(tar));
       acc(LT_INS_TARWAIT, tt);
       fence_proxy_async();
@@ -420,7 +489,7 @@ struct OpL {
   // BGPQ_DELETEMIN (Alg.2 + Alg.3).  call_n > 0: deletemin-call mode (size and output slot
   // from the per-call ticket); else `size` and `ok/ov` are given.  Returns #keys written.
   // =====================================================================================
-  __device__ u32 deletemin(u32* ok, u32* ov, u32 size, u64 call_n, ull* lin_out) {
+  __device__ __forceinline__ u32 deletemin(u32* ok, u32* ov, u32 size, u64 call_n, ull* lin_out) {
     const int tid = threadIdx.x;
     enum : u32 { P_EMPTY = 0, P_EXTRACT = 1, P_PBUF = 2, P_REFILL = 3 };
     tmerge = LT_DEL_MERGE; tstore = LT_DEL_STORE;
@@ -434,18 +503,18 @@ struct OpL {
       acc(LT_DEL_ROOTACQ, t_del);
       t_root = now();
       fence_proxy_async();
-      const ull lin = lin_get();
-      lin_set(lin + 1);
-      if (lin_out) *lin_out = lin;
+      const Hdr h = hdr_load();
+      lin_set(h.lin + 1);
+      if (lin_out) *lin_out = h.lin;
       u32 cno = 0;
       if (call_n) {
-        cno = hget(H_CALL);
+        cno = h.call;
         hset(H_CALL, cno + 1);
         const u64 rem = call_n - (u64)cno * K;
         size = (u32)(rem < (u64)K ? rem : (u64)K);
       }
-      const u32 hs = hget(H_HS), rs = hget(H_RS), ps = hget(H_PS);
-      const u32 pbmin = ld_relaxed(&H.meta[0].kmin);
+      const u32 hs = h.hs, rs = h.rs, ps = h.ps;
+      const u32 pbmin = h.pbmin;
       const u32 path = hs == 0 ? P_EMPTY : size < rs ? P_EXTRACT : hs == 1 ? P_PBUF : P_REFILL;
       int sr = -1, stt = -1;
       if (rs > 0 && path != P_EMPTY) {  // stage the root (its keys are output first)
@@ -461,6 +530,7 @@ struct OpL {
         st[S_DEL_REFILL]++;
         st_relaxed(stp(1), ST_EMPTY);  // l.31
         hset(H_HS, hs - 1);
+        if (BGPQ_PREFETCH && hs - 1 >= 2) prefetch_l2(hs - 1);  // the next DELETEMIN's refill node
         stt = alloc();
         post_t(tar, stt, rs > 0 ? 1u : 0u);  // l.6-12 by agent T
         if (tar >= 4) {  // LOCK(l); LOCK(r) of the root concurrently (agent P)
@@ -474,8 +544,10 @@ struct OpL {
       ctl->b[0] = hs; ctl->b[1] = rs; ctl->b[2] = ps; ctl->b[3] = pbmin;
       ctl->b[4] = cno; ctl->b[5] = size; ctl->b[6] = path;
       ctl->b[10] = (u32)sr; ctl->b[11] = (u32)stt;
+      tmark = t_root;
     }
     cta_bar<NT>();
+    mark(LT_R1);
     const u32 hs = ctl->b[0], rs = ctl->b[1], ps = ctl->b[2], pbmin = ctl->b[3];
     const u32 path = ctl->b[6];
     size = ctl->b[5];
@@ -543,6 +615,7 @@ struct OpL {
     mbar_wait(&ctl->tbar, tphase);  // agent T staged the refill keys (tar's, or a MARKED insert's)
     tphase ^= 1u;
     acc(LT_DEL_TWAIT, t_tw);
+    mark(LT_R2);
     int R = (int)ctl->b[11];
     cta_bar<NT>();
     if (tid == 0) {
@@ -578,6 +651,7 @@ struct OpL {
     for (;;) {
       const u32 l = 2u * cur, r = 2u * cur + 1u;  // l.2 (R7)
       wait_p(LT_DEL_PWAIT);  // l.3: LOCK(l); LOCK(r) — done by agent P, children staged
+      if (cur == 1) mark(LT_R3);
       if (tid == 0) {
         const u32 le = l <= H.cap, re = r <= H.cap;
         const u32 al = le && ctl->p_st[0] == ST_AVAIL;  // R5
@@ -654,17 +728,21 @@ struct OpL {
       if (lr == 2) {  // l.10: (Heap[y], Heap[x]) <- SORT_SPLIT(Heap[l], Heap[r])
         const int a = (int)ctl->b[10], b = (int)ctl->b[11];
         merge_split(SL, K, SRr, K, K, a, b);
+        if (cur == 1) mark(LT_R4);
         store(x, b);
         if (tid == 0) {
           set_minmax(x, BK(b)[0], BK(b)[K - 1]);
-          lock_release(lk(x));  // l.11: UNLOCK(x)
+          ctl->b[16] = x;  // l.11: UNLOCK(x) — released with cur below (one fence)
+          if (!BGPQ_JOINT_RELEASE) { lock_release(lk(x)); ctl->b[16] = 0; }
           free_slot(b); free_slot(SL); free_slot(SRr);
         }
+        if (cur == 1) mark(LT_R5);
         Y = a;
       } else {  // no data moves between l and r (or only y is AVAIL)
         Y = (y == l) ? SL : SRr;
         if (tid == 0) {
-          if (x == l ? le : re) lock_release(lk(x));
+          ctl->b[16] = (x == l ? le : re) ? x : 0u;
+          if (!BGPQ_JOINT_RELEASE && ctl->b[16]) { lock_release(lk(x)); ctl->b[16] = 0; }
           free_slot(y == l ? SRr : SL);
         }
       }
@@ -693,6 +771,7 @@ struct OpL {
           shift(src, C2, remained, K - remained);
         }
         store(1, src);
+        mark(LT_R6);
         if (tid == 0) {
           hset(H_RS, K - remained);
           if (remained < (u32)K) set_minmax(1, BK(src)[0], BK(src)[K - remained - 1]);
@@ -705,8 +784,8 @@ struct OpL {
       if (tid == 0) {
         free_slot(C2);
         if (cur == 1) while (ld_acq_cta(&ctl->t_done) != ctl->t_req) {}  // the take is done
-        lock_release(lk(cur));  // l.14: UNLOCK(cur)
-        if (cur == 1) acc(LT_DEL_ROOTHOLD, t_root);
+        release_locks(cur, ctl->b[16]);  // l.14: UNLOCK(cur) (and l.11's UNLOCK(x))
+        if (cur == 1) { acc(LT_DEL_ROOTHOLD, t_root); mark(LT_R7); }
         if (timing && tid == 0) tm[LT_DEL_LEVELS]++;
       }
       cur = y;  // l.15
@@ -731,7 +810,7 @@ struct OpL {
 
 // ---- the lock warp: lane 0 = agent P, lane 1 = agent T
 template <int K, bool V, int NT>
-__device__ void lock_warp(OpL<K, V, NT>& op) {
+__device__ __forceinline__ void lock_warp(OpL<K, V, NT>& op) {
   LCtl* c = op.ctl;
   const int lane = threadIdx.x & 31;
   const u32 NB = K * 4u;
@@ -781,6 +860,13 @@ __device__ void lock_warp(OpL<K, V, NT>& op) {
       seen = r;
       const u32 n = c->t_node;
       const int s = (int)c->t_slot;
+      if (c->t_kind == 1u) {  // Alg.1 l.5-6
+        lock_acquire(op.lk(n));
+        st_relaxed(op.stp(n), ST_TARGET);
+        lock_release(op.lk(n));
+        st_rel_cta(&c->t_done, seen);
+        continue;
+      }
       const ull t0 = op.timing ? clock64() : 0;
       lock_acquire(op.lk(n));  // l.6: LOCK(tar)
       if (op.timing) op.tm[LT_T_LOCKWAIT] += clock64() - t0;
@@ -826,13 +912,15 @@ __global__ void __launch_bounds__(NT + 32, 1) bgpq_locks_kernel(HeapArgs H, Call
   OpL<K, V, NT> op;
   op.H = H;
   op.ctl = ctl;
-  op.sk = reinterpret_cast<u32*>(smem_raw + 512);
+  op.sk = reinterpret_cast<u32*>(smem_raw + LCTL_BYTES);
   op.sv = op.sk + LSLOT * K;
-  op.mphase = 0; op.pphase[0] = op.pphase[1] = 0; op.tphase = 0; op.pb = 0;
-  for (int i = 0; i < NSTAT; ++i) op.st[i] = 0;
+  op.mphase = 0; op.pph = 0; op.tphase = 0; op.pb = 0;
+  op.st = ctl->st;
+  op.tm = ctl->tm;
   op.timing = (C.debug & 8u) != 0;
-  for (int i = 0; i < LT_N; ++i) op.tm[i] = 0;
   if (threadIdx.x == 0) {
+    for (int i = 0; i < NSTAT; ++i) ctl->st[i] = 0;
+    for (int i = 0; i < 32; ++i) ctl->tm[i] = 0;
     mbar_init(&ctl->bar, 1);
     mbar_init(&ctl->pbar[0], 1);
     mbar_init(&ctl->pbar[1], 1);
@@ -846,7 +934,7 @@ __global__ void __launch_bounds__(NT + 32, 1) bgpq_locks_kernel(HeapArgs H, Call
     lock_warp<K, V, NT>(op);
     if (op.timing) {
       ull* tms = reinterpret_cast<ull*>(H.hdr + H_TIME);
-      for (int i = LT_P_LOCKWAIT; i < LT_N; ++i)
+      for (int i = LT_P_LOCKWAIT; i < LT_R1; ++i)
         if (op.tm[i]) atomicAdd(tms + i, op.tm[i]);
     }
     return;
@@ -857,30 +945,46 @@ __global__ void __launch_bounds__(NT + 32, 1) bgpq_locks_kernel(HeapArgs H, Call
     const u64 j = ctl->op;
     cta_bar<NT>();
     if (j >= C.n_ops) break;
+    // one call site per operation type (both are force-inlined: no local-memory copy of op)
+    bool ins;
+    const u32* ik = nullptr;
+    const u32* iv = nullptr;
+    u32* ok = C.out_k;
+    u32* ov = C.out_v;
+    u32 size = 0;
+    u64 call_n = 0;
+    ull* lt = nullptr;
     if (C.mode == MODE_INSERT) {
+      ins = true;
       const u64 off = j * (u64)K;
       const u64 rem = C.n - off;
-      const u32 size = (u32)(rem < (u64)K ? rem : (u64)K);
-      op.insert(C.in_k + off, C.in_v ? C.in_v + off : nullptr, size, nullptr);
+      size = (u32)(rem < (u64)K ? rem : (u64)K);
+      ik = C.in_k + off;
+      iv = C.in_v ? C.in_v + off : nullptr;
     } else if (C.mode == MODE_DELETEMIN) {
-      const u32 cnt = op.deletemin(C.out_k, C.out_v, 0, C.n, nullptr);
+      ins = false;
+      call_n = C.n;
+    } else {
+      ins = C.op_types[j] == 0;
+      size = C.op_sizes[j];
+      lt = C.lin_ticket ? C.lin_ticket + j : nullptr;
+      if (ins) {
+        const u64 off = C.in_off[j];
+        ik = C.in_k + off;
+        iv = C.in_v ? C.in_v + off : nullptr;
+      } else {
+        ok = C.out_k + j * (u64)K;
+        ov = C.out_v ? C.out_v + j * (u64)K : nullptr;
+      }
+    }
+    if (ins) {
+      op.insert(ik, iv, size, lt);
+    } else {
+      const u32 cnt = op.deletemin(ok, ov, size, call_n, lt);
       if (threadIdx.x == 0) {
         op.st[S_KEYS_OUT] += cnt;
-        if (C.d_count && cnt) atomicAdd(C.d_count, (ull)cnt);
-      }
-    } else {
-      const u32 size = C.op_sizes[j];
-      ull* lt = C.lin_ticket ? C.lin_ticket + j : nullptr;
-      if (C.op_types[j] == 0) {
-        const u64 off = C.in_off[j];
-        op.insert(C.in_k + off, C.in_v ? C.in_v + off : nullptr, size, lt);
-      } else {
-        const u32 cnt = op.deletemin(C.out_k + j * (u64)K, C.out_v ? C.out_v + j * (u64)K : nullptr,
-                                     size, 0, lt);
-        if (threadIdx.x == 0) {
-          op.st[S_KEYS_OUT] += cnt;
-          C.op_count[j] = cnt;
-        }
+        if (C.mode == MODE_MIXED) C.op_count[j] = cnt;
+        else if (C.d_count && cnt) atomicAdd(C.d_count, (ull)cnt);
       }
     }
   }
@@ -891,7 +995,8 @@ __global__ void __launch_bounds__(NT + 32, 1) bgpq_locks_kernel(HeapArgs H, Call
       if (op.st[i]) atomicAdd(stat + i, op.st[i]);
     if (op.timing) {
       ull* tms = reinterpret_cast<ull*>(H.hdr + H_TIME);
-      for (int i = 0; i < LT_P_LOCKWAIT; ++i)
+      for (int i = 0; i < LT_N; ++i)
+        if (i < LT_P_LOCKWAIT || i >= LT_R1)
         if (op.tm[i]) atomicAdd(tms + i, op.tm[i]);
     }
   }
@@ -899,7 +1004,7 @@ __global__ void __launch_bounds__(NT + 32, 1) bgpq_locks_kernel(HeapArgs H, Call
 
 template <int K, bool V>
 constexpr size_t locks_smem_bytes() {
-  return 512 + (size_t)LSLOT * K * 4 * (V ? 2 : 1);
+  return LCTL_BYTES + (size_t)LSLOT * K * 4 * (V ? 2 : 1);
 }
 
 }  // namespace bgpqd
