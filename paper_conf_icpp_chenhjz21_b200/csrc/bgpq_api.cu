@@ -12,6 +12,7 @@
 
 #include "../../include/bgpq.h"
 #include "bgpq_locks.cuh"
+#include "bgpq_pipe.cuh"
 #include "bgpq_server.cuh"
 
 using namespace bgpqd;
@@ -52,6 +53,9 @@ struct bgpq {
   int occ = 0;         // co-resident CTAs per SM for this K
   int grid_req = 0;    // 0 auto, else exact
   SrvArgs srv{};           // server-mode rings and control words (device)
+  PipeArgs pipe{};         // insert-pipeline rings (allocated at the first pipelined insert)
+  bool pipe_ok = false;
+  int pipe_grid = 0;
   bool srv_ok = false;
   int srv_grid = 0;
   u32* stage_k = nullptr;  // staging for the *_host calls
@@ -99,6 +103,23 @@ struct KernelInfo {
     return cudaGetLastError();
   }
   static int srv_top_nodes() { return SrvShape<K, V, NT>::NTOP; }
+  static int pipe_occupancy(int* out_occ) {
+    auto kern = bgpq_ins_pipe_kernel<K, V, NT>;
+    const size_t smem = pipe_smem_bytes<K, V>();
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return -1;
+    int occ = 0;
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, NT, smem);
+    if (e != cudaSuccess) return -1;
+    *out_occ = occ;
+    return 0;
+  }
+  static cudaError_t pipe_launch(int grid, const HeapArgs& H, const PipeArgs& P, const CallArgs& C,
+                                 cudaStream_t s) {
+    bgpq_ins_pipe_kernel<K, V, NT><<<grid, NT, pipe_smem_bytes<K, V>(), s>>>(H, P, C);
+    g_launches.fetch_add(1);
+    return cudaGetLastError();
+  }
 };
 
 int occupancy_for(u32 K, bool V, int* occ) {
@@ -182,6 +203,39 @@ cudaError_t srv_launch_for(u32 K, bool V, int grid, const HeapArgs& H, const Cal
 #undef BGPQ_CASE
 }
 
+int pipe_occupancy_for(u32 K, bool V, int* occ) {
+#define BGPQ_CASE(KK)                                                                        \
+  case KK:                                                                                   \
+    return V ? KernelInfo<KK, true>::pipe_occupancy(occ) : KernelInfo<KK, false>::pipe_occupancy(occ);
+  switch (K) {
+    BGPQ_CASE(64)
+    BGPQ_CASE(128)
+    BGPQ_CASE(256)
+    BGPQ_CASE(512)
+    BGPQ_CASE(1024)
+    default:
+      return -1;
+  }
+#undef BGPQ_CASE
+}
+
+cudaError_t pipe_launch_for(u32 K, bool V, int grid, const HeapArgs& H, const PipeArgs& P, const CallArgs& C,
+                            cudaStream_t s) {
+#define BGPQ_CASE(KK)                                                                        \
+  case KK:                                                                                   \
+    return V ? KernelInfo<KK, true>::pipe_launch(grid, H, P, C, s) : KernelInfo<KK, false>::pipe_launch(grid, H, P, C, s);
+  switch (K) {
+    BGPQ_CASE(64)
+    BGPQ_CASE(128)
+    BGPQ_CASE(256)
+    BGPQ_CASE(512)
+    BGPQ_CASE(1024)
+    default:
+      return cudaErrorInvalidValue;
+  }
+#undef BGPQ_CASE
+}
+
 bool valid_K(u32 K) { return K == 64 || K == 128 || K == 256 || K == 512 || K == 1024; }
 
 HeapArgs heap_args(const bgpq* q) {
@@ -201,10 +255,57 @@ int grid_for(const bgpq* q, u64 n_ops) {
   return (int)std::max(1LL, g);
 }
 
+u32 depth_host(u32 i) {
+  u32 d = 0;
+  while (i > 1) { i >>= 1; ++d; }
+  return d;
+}
+
 bool server_mode(const bgpq* q) { return (q->flags & BGPQ_FLAG_SERVER) && !(q->flags & BGPQ_FLAG_SERIAL); }
+
+// Insert-only calls in the default execution run as a level pipeline (bgpq_pipe.cuh).
+bool pipe_mode(const bgpq* q) {
+  return !(q->flags & (BGPQ_FLAG_SERIAL | BGPQ_FLAG_LOCKS | BGPQ_FLAG_SERVER));
+}
+
+bool ensure_pipe(bgpq* q) {
+  if (q->pipe_ok) return true;
+  const bool V = (q->flags & BGPQ_FLAG_VALUES) != 0;
+  const u32 depth = depth_host(q->cap_nodes);
+  int occ = 0;
+  if (pipe_occupancy_for(q->K, V, &occ) != 0 || occ < 1) return false;
+  const int grid = q->sm_count;  // one CTA per SM, all co-resident
+  if ((int)depth + 2 > grid || depth >= PIPE_MAXL) return false;
+  PipeArgs& P = q->pipe;
+  const size_t kb = (size_t)q->K * sizeof(u32);
+  bool ok = cudaMalloc(&P.ctl, PC_WORDS * sizeof(u32)) == cudaSuccess;
+  ok = ok && cudaMalloc(&P.sbk, PIPE_NSB * kb) == cudaSuccess;
+  ok = ok && cudaMalloc(&P.sready, PIPE_NSB * sizeof(u32)) == cudaSuccess;
+  ok = ok && cudaMalloc(&P.rk, (size_t)PIPE_MAXL * PIPE_NL * kb) == cudaSuccess;
+  ok = ok && cudaMalloc(&P.rhdr, (size_t)PIPE_MAXL * PIPE_NL * 4 * sizeof(u32)) == cudaSuccess;
+  ok = ok && cudaMalloc(&P.rflag, (size_t)PIPE_MAXL * PIPE_NL * sizeof(u32)) == cudaSuccess;
+  if (V) {
+    ok = ok && cudaMalloc(&P.sbv, PIPE_NSB * kb) == cudaSuccess;
+    ok = ok && cudaMalloc(&P.rv, (size_t)PIPE_MAXL * PIPE_NL * kb) == cudaSuccess;
+  }
+  P.depth = depth;
+  q->pipe_grid = grid;
+  q->pipe_ok = ok;
+  return ok;
+}
 
 int run_call(bgpq* q, const CallArgs& C, cudaStream_t s) {
   const bool V = (q->flags & BGPQ_FLAG_VALUES) != 0;
+  if (C.mode == MODE_INSERT && pipe_mode(q)) {
+    if (!ensure_pipe(q)) return fail(BGPQ_ENOMEM);
+    const PipeArgs& P = q->pipe;
+    bool ok = cudaMemsetAsync(P.ctl, 0, PC_WORDS * sizeof(u32), s) == cudaSuccess;
+    ok = ok && cudaMemsetAsync(P.sready, 0, PIPE_NSB * sizeof(u32), s) == cudaSuccess;
+    ok = ok && cudaMemsetAsync(P.rflag, 0, (size_t)PIPE_MAXL * PIPE_NL * sizeof(u32), s) == cudaSuccess;
+    if (!ok) return fail(BGPQ_ECUDA);
+    if (pipe_launch_for(q->K, V, q->pipe_grid, heap_args(q), P, C, s) != cudaSuccess) return fail(BGPQ_ECUDA);
+    return BGPQ_OK;
+  }
   if (server_mode(q)) {
     // reset the per-call control words, publication flags, gate tickets and lend counters
     const int ntop = srv_top_for(q->K, V);
@@ -319,6 +420,9 @@ void bgpq_destroy(bgpq_t* q) {
   SrvArgs& A = q->srv;
   u32* bufs[] = {A.ctl, A.task, A.task_pub, A.payk, A.payv, A.sbk, A.sbv, A.sready, A.serving, A.ret, A.mailk, A.mailv};
   for (u32* b : bufs) cudaFree(b);
+  PipeArgs& P = q->pipe;
+  u32* pbufs[] = {P.ctl, P.sbk, P.sbv, P.sready, P.rk, P.rv, P.rhdr, P.rflag};
+  for (u32* b : pbufs) cudaFree(b);
   delete q;
 }
 

@@ -33,7 +33,13 @@ def _gpu_inv(q):
 # --------------------------------------------------------------------------------------
 # phased insert-all then deletemin-all: output == sorted(input) (closed form, §8(c))
 # --------------------------------------------------------------------------------------
-MODES = ["server", "locks"]
+MODES = ["default", "locks", "server"]
+
+
+def _mode(mode):
+    """default: INSERT calls as the level pipeline + lock-ahead DELETEMIN; locks: paper-literal
+    per-node locks for every call; server: root-server execution."""
+    return {"locks": mode == "locks", "server": mode == "server"}
 
 
 @pytest.mark.parametrize("mode", MODES)
@@ -45,7 +51,7 @@ def test_phased_sorted(K, dist, mode):
         n = 300 * K + 37  # deeper than the on-chip levels for every K
     keys = synth.keys(n, seed=synth.SEEDS["C3"], dist=dist)
     vals = synth.values(n)
-    q = pkg.BGPQ(capacity=n, K=K, values=True, server=(mode == "server"))
+    q = pkg.BGPQ(capacity=n, K=K, values=True, **_mode(mode))
     q.insert(_dev(keys), _dev(vals))
     assert q.size() == n
     assert _gpu_inv(q) == (0, 0)
@@ -103,6 +109,25 @@ def test_serialized_layout_bitexact_phased(K):
     want = np.concatenate([seq.deletemin(K)[0] for _ in range(37)])
     assert np.array_equal(_host(ok), want)
     _compare_layout(q, seq)
+
+
+@pytest.mark.parametrize("K", [64, 1024])
+@pytest.mark.parametrize("values", [False, True])
+def test_pipelined_insert_layout_bitexact(K, values):
+    """INSERT calls run as a level pipeline that applies the batches at every node in call
+    order: the heap after the call equals the sequential Alg.1 model node for node, including
+    a second call on a non-empty heap with a partial batch and a non-empty pBuffer."""
+    n1, n2 = 37 * K + 5, 50 * K + 11
+    keys = synth.keys(n1 + n2, seed=9, dist="dups")
+    q = pkg.BGPQ(capacity=n1 + n2, K=K, values=values)
+    seq = oracle.SeqBGPQ(K, q.slots() - 1)
+    for a, b in ((0, n1), (n1, n1 + n2)):
+        q.insert(_dev(keys[a:b]), _dev(synth.values(b - a)) if values else None)
+        for off in range(a, b, K):
+            seq.insert(keys[off:min(off + K, b)])
+        _compare_layout(q, seq)
+    ok, _ = q.deletemin(n1 + n2)
+    assert np.array_equal(_host(ok), np.sort(keys))
 
 
 def _mixed_inputs(types, sizes, K, seed, dist="uniform"):
@@ -183,7 +208,7 @@ def test_concurrent_mixed_replay(K, p_ins, partial, mode):
         types, _ = synth.random_ops(n_ops, K, seed=41 + K, p_insert=p_ins)
         sizes = np.full(n_ops, K, np.uint32)
     keys, in_off = _mixed_inputs(types, sizes, K, seed=43)
-    q = pkg.BGPQ(capacity=len(keys) + K, K=K, values=True, server=(mode == "server"))
+    q = pkg.BGPQ(capacity=len(keys) + K, K=K, values=True, **_mode(mode))
     outk, outv, cnt, lin = _run_mixed(q, types, sizes, keys, in_off)
     ref = _replay_check(types, sizes, keys, in_off, outk, outv, cnt, lin)
     for j in np.nonzero(types == 1)[0]:
@@ -200,7 +225,7 @@ def test_concurrent_pairs_with_prefill_replay(mode):
     """Utilisation shape: prefill, then insert/deletemin pairs on all CTAs."""
     K = 64
     pre = synth.keys(1 << 17, seed=50)
-    q = pkg.BGPQ(capacity=(1 << 18) + 4096 * K, K=K, values=True, server=(mode == "server"))
+    q = pkg.BGPQ(capacity=(1 << 18) + 4096 * K, K=K, values=True, **_mode(mode))
     q.insert(_dev(pre), _dev(synth.values(len(pre))))
     types, sizes = synth.mixed_ops(3000, K, seed=51, partial=True)
     keys, in_off = _mixed_inputs(types, sizes, K, seed=52)
@@ -219,7 +244,7 @@ def test_marked_handoff_replay(mode):
         types, _ = synth.random_ops(3000, K, seed=60 + seed, p_insert=0.5)
         sizes = np.full(len(types), K, np.uint32)
         keys, in_off = _mixed_inputs(types, sizes, K, seed=70 + seed)
-        q = pkg.BGPQ(capacity=len(keys) + K, K=K, values=True, server=(mode == "server"))
+        q = pkg.BGPQ(capacity=len(keys) + K, K=K, values=True, **_mode(mode))
         outk, outv, cnt, lin = _run_mixed(q, types, sizes, keys, in_off)
         _replay_check(types, sizes, keys, in_off, outk, outv, cnt, lin)
         assert _gpu_inv(q) == (0, 0)
@@ -275,7 +300,7 @@ def test_full_size_c2_properties(mode):
     n, K = 1 << 27, 1024
     keys = synth.keys(n, seed=synth.SEEDS["C2"])
     dk = _dev(keys)
-    q = pkg.BGPQ(capacity=n, K=K, values=False, server=(mode == "server"))
+    q = pkg.BGPQ(capacity=n, K=K, values=False, **_mode(mode))
     q.insert(dk)
     assert q.size() == n
     ok, _ = q.deletemin(n)
