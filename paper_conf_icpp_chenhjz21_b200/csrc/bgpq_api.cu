@@ -14,6 +14,7 @@
 #include "bgpq_locks.cuh"
 #include "bgpq_pipe.cuh"
 #include "bgpq_server.cuh"
+#include "bgpq_dtop.cuh"
 
 using namespace bgpqd;
 
@@ -58,6 +59,8 @@ struct bgpq {
   int pipe_grid = 0;
   bool srv_ok = false;
   int srv_grid = 0;
+  DtArgs dt{};             // deletemin top-CTA execution: walker task list (bgpq_dtop.cuh)
+  bool dt_ok = false;
   u32* stage_k = nullptr;  // staging for the *_host calls
   u32* stage_v = nullptr;
   u64* stage_cnt = nullptr;
@@ -99,6 +102,23 @@ struct KernelInfo {
   static cudaError_t srv_launch(int grid, const HeapArgs& H, const CallArgs& C, const SrvArgs& A,
                                 cudaStream_t s) {
     bgpq_srv_kernel<K, V, NT><<<grid, NT + 32, SrvShape<K, V, NT>::smem, s>>>(H, C, A);
+    g_launches.fetch_add(1);
+    return cudaGetLastError();
+  }
+  static cudaError_t dt_launch(int grid, const HeapArgs& H, const CallArgs& C, const DtArgs& D, cudaStream_t s) {
+    static bool attr = false;
+    auto kern = bgpq_dtop_kernel<K, V>;
+    const size_t smem = dt_smem_bytes<K, V>();
+    if (!attr) {
+      cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+      if (e != cudaSuccess) return e;
+      int occ = 0;
+      e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, DT_BLOCK, smem);
+      if (e != cudaSuccess) return e;
+      if (occ < 1) return cudaErrorLaunchOutOfResources;
+      attr = true;
+    }
+    kern<<<grid, DT_BLOCK, smem, s>>>(H, C, D);
     g_launches.fetch_add(1);
     return cudaGetLastError();
   }
@@ -203,6 +223,23 @@ cudaError_t srv_launch_for(u32 K, bool V, int grid, const HeapArgs& H, const Cal
 #undef BGPQ_CASE
 }
 
+cudaError_t dt_launch_for(u32 K, bool V, int grid, const HeapArgs& H, const CallArgs& C, const DtArgs& D,
+                          cudaStream_t s) {
+#define BGPQ_CASE(KK)                                                                        \
+  case KK:                                                                                   \
+    return V ? KernelInfo<KK, true>::dt_launch(grid, H, C, D, s) : KernelInfo<KK, false>::dt_launch(grid, H, C, D, s);
+  switch (K) {
+    BGPQ_CASE(64)
+    BGPQ_CASE(128)
+    BGPQ_CASE(256)
+    BGPQ_CASE(512)
+    BGPQ_CASE(1024)
+    default:
+      return cudaErrorInvalidValue;
+  }
+#undef BGPQ_CASE
+}
+
 int pipe_occupancy_for(u32 K, bool V, int* occ) {
 #define BGPQ_CASE(KK)                                                                        \
   case KK:                                                                                   \
@@ -294,8 +331,39 @@ bool ensure_pipe(bgpq* q) {
   return ok;
 }
 
+// Deletemin-only calls in the default execution: top CTA + walkers (bgpq_dtop.cuh).
+// BGPQ_DEBUG bit 16 routes them to the per-op lock execution instead (A/B comparisons).
+bool dt_mode(const bgpq* q) { return pipe_mode(q) && !(g_debug & 16u); }
+
+bool ensure_dt(bgpq* q) {
+  if (q->dt_ok) return true;
+  DtArgs& D = q->dt;
+  const size_t n = (size_t)q->cap_nodes + 2;
+  bool ok = cudaMalloc(&D.task_node, n * sizeof(u32)) == cudaSuccess;
+  ok = ok && cudaMalloc(&D.task_seq, n * sizeof(u32)) == cudaSuccess;
+  ok = ok && cudaMalloc(&D.ctl, 32 * sizeof(u32)) == cudaSuccess;
+  ok = ok && cudaMemset(D.task_seq, 0, n * sizeof(u32)) == cudaSuccess;
+  ok = ok && cudaMemset(D.ctl, 0, 32 * sizeof(u32)) == cudaSuccess;
+  D.epoch = 0;
+  q->dt_ok = ok;
+  return ok;
+}
+
 int run_call(bgpq* q, const CallArgs& C, cudaStream_t s) {
   const bool V = (q->flags & BGPQ_FLAG_VALUES) != 0;
+  if (C.mode == MODE_DELETEMIN && dt_mode(q)) {
+    if (!ensure_dt(q)) return fail(BGPQ_ENOMEM);
+    DtArgs& D = q->dt;
+    D.epoch += 1;
+    if (D.epoch == 0) {  // wrapped: clear the stale epochs
+      D.epoch = 1;
+      if (cudaMemsetAsync(D.task_seq, 0, ((size_t)q->cap_nodes + 2) * sizeof(u32), s) != cudaSuccess)
+        return fail(BGPQ_ECUDA);
+    }
+    if (cudaMemsetAsync(D.ctl, 0, 2 * sizeof(u32), s) != cudaSuccess) return fail(BGPQ_ECUDA);
+    if (dt_launch_for(q->K, V, q->sm_count, heap_args(q), C, D, s) != cudaSuccess) return fail(BGPQ_ECUDA);
+    return BGPQ_OK;
+  }
   if (C.mode == MODE_INSERT && pipe_mode(q)) {
     if (!ensure_pipe(q)) return fail(BGPQ_ENOMEM);
     const PipeArgs& P = q->pipe;
@@ -420,6 +488,9 @@ void bgpq_destroy(bgpq_t* q) {
   SrvArgs& A = q->srv;
   u32* bufs[] = {A.ctl, A.task, A.task_pub, A.payk, A.payv, A.sbk, A.sbv, A.sready, A.serving, A.ret, A.mailk, A.mailv};
   for (u32* b : bufs) cudaFree(b);
+  cudaFree(q->dt.task_node);
+  cudaFree(q->dt.task_seq);
+  cudaFree(q->dt.ctl);
   PipeArgs& P = q->pipe;
   u32* pbufs[] = {P.ctl, P.sbk, P.sbv, P.sready, P.rk, P.rv, P.rhdr, P.rflag};
   for (u32* b : pbufs) cudaFree(b);

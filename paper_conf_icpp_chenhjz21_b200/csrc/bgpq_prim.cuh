@@ -96,6 +96,13 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, u32 bytes, 
       "l"(src), "r"(bytes), "r"(smem_addr(bar)) : "memory");
 }
 
+// TMA bulk copy shared -> global (bulk_group completion; the issuing thread waits with
+// cp.async.bulk.wait_group[.read])
+__device__ __forceinline__ void bulk_s2g(void* dst, const void* src, u32 bytes) {
+  asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst), "r"(smem_addr(src)),
+               "r"(bytes) : "memory");
+}
+
 // CTA barrier over the NT compute threads only (named barrier 1): the server CTA runs an
 // extra helper warp that must not take part in the compute barriers.
 template <int NT>
@@ -345,8 +352,9 @@ __device__ __forceinline__ void bitonic_sort_regs(T (&c)[VT]) {
   }
 }
 
+// grp_merge_win: the same merge executed by a group of NTM threads, t = index in the group
 template <int KMAX, int NTM, bool V>
-__device__ __forceinline__ void cta_merge_win(const u32* __restrict__ zk, const u32* __restrict__ zv,
+__device__ __forceinline__ void grp_merge_win(const int t, const u32* __restrict__ zk, const u32* __restrict__ zv,
                                               int na, const u32* __restrict__ wk,
                                               const u32* __restrict__ wv, int nb, int ma,
                                               u32* __restrict__ xk, u32* __restrict__ xv,
@@ -354,7 +362,6 @@ __device__ __forceinline__ void cta_merge_win(const u32* __restrict__ zk, const 
   constexpr int VT = (2 * KMAX) / NTM;
   static_assert(VT >= 2 && (VT & (VT - 1)) == 0 && VT * NTM == 2 * KMAX, "VT must be a power of two");
   constexpr int LOG = Log2Ceil<KMAX + 1>::v;
-  const int t = threadIdx.x;
   if (t >= NTM) return;
   const int N = na + nb;
   const int d = t * VT;
@@ -439,6 +446,15 @@ __device__ __forceinline__ void cta_merge_win(const u32* __restrict__ zk, const 
   }
 }
 
+template <int KMAX, int NTM, bool V>
+__device__ __forceinline__ void cta_merge_win(const u32* __restrict__ zk, const u32* __restrict__ zv,
+                                              int na, const u32* __restrict__ wk,
+                                              const u32* __restrict__ wv, int nb, int ma,
+                                              u32* __restrict__ xk, u32* __restrict__ xv,
+                                              u32* __restrict__ yk, u32* __restrict__ yv) {
+  grp_merge_win<KMAX, NTM, V>((int)threadIdx.x, zk, zv, na, wk, wv, nb, ma, xk, xv, yk, yv);
+}
+
 // ----------------------------------------------------------------------------------------
 // SORT_SPLIT by warp-cooperative merge path (v4, the hot-path merge).
 // Warp w of the first NW warps produces the OW = 2*KMAX/NW consecutive outputs [D0, D0+OW)
@@ -488,7 +504,7 @@ __device__ __forceinline__ int warp_corank(const u32* __restrict__ zk, int na, c
 }
 
 template <int KMAX, int NW, bool V>
-__device__ __forceinline__ void cta_merge_warp(const u32* __restrict__ zk, const u32* __restrict__ zv,
+__device__ __forceinline__ void grp_merge_warp(const int warp, const u32* __restrict__ zk, const u32* __restrict__ zv,
                                                int na, const u32* __restrict__ wk,
                                                const u32* __restrict__ wv, int nb, int ma,
                                                u32* __restrict__ xk, u32* __restrict__ xv,
@@ -497,7 +513,7 @@ __device__ __forceinline__ void cta_merge_warp(const u32* __restrict__ zk, const
   constexpr int E = OW / 32;
   static_assert(E >= 1 && (E & (E - 1)) == 0 && OW * NW == 2 * KMAX, "E must be a power of two");
   using T = typename std::conditional<V, u64, u32>::type;
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int lane = threadIdx.x & 31;
   if (warp >= NW) return;
   const int N = na + nb;
   const int D0 = warp * OW;
@@ -558,6 +574,15 @@ __device__ __forceinline__ void cta_merge_warp(const u32* __restrict__ zk, const
       else { yk[o - ma] = key; if (V) yv[o - ma] = val; }
     }
   }
+}
+
+template <int KMAX, int NW, bool V>
+__device__ __forceinline__ void cta_merge_warp(const u32* __restrict__ zk, const u32* __restrict__ zv,
+                                               int na, const u32* __restrict__ wk,
+                                               const u32* __restrict__ wv, int nb, int ma,
+                                               u32* __restrict__ xk, u32* __restrict__ xv,
+                                               u32* __restrict__ yk, u32* __restrict__ yv) {
+  grp_merge_warp<KMAX, NW, V>((int)(threadIdx.x >> 5), zk, zv, na, wk, wv, nb, ma, xk, xv, yk, yv);
 }
 
 // The SORT_SPLIT used on the hot path: register-window merge path with VT = 4 outputs per
