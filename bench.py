@@ -165,7 +165,10 @@ def _config(args):
                          f"then deletemin all, K={args.K}, {'key+value' if args.values else 'keys only'} "
                          f"(w={w} B)"),
             "n_keys": 1 << args.n_log2, "K": args.K, "w_bytes": w, "dist": args.dist,
-            "threads_per_cta": 512, "execution": args.mode, "l2": f"inputs and heap ({(1 << args.n_log2) * w * 3 >> 20} MiB) "
+            "execution": ({"insert": "level pipeline (bgpq_ins_pipe_kernel, one CTA per heap level)",
+                           "deletemin": "top CTA + walker CTAs (bgpq_dtop_kernel)"} if args.mode == "locks" else
+                          {"insert": "root-server (bgpq_srv_kernel)", "deletemin": "root-server (bgpq_srv_kernel)"}),
+            "l2": f"inputs and heap ({(1 << args.n_log2) * w * 3 >> 20} MiB) "
                                           "larger than the 126 MB L2; no flush"}
 
 
@@ -204,7 +207,8 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--profile-steps", type=int, default=0, help="ncu mode: run N untimed steps and exit")
     ap.add_argument("--mode", default="locks", choices=["locks", "server"],
-                    help="execution: paper-literal per-node locks on all CTAs, or root-server CTA")
+                    help="execution: default (insert level pipeline + deletemin top CTA with walkers "
+                         "taking the paper's per-node locks), or the root-server CTA")
     args = ap.parse_args()
     world, rank, local = _dist_setup()
 
@@ -327,7 +331,7 @@ def main():
             "config": _config(args),
             "parallelism": "replicas only (one linearizable heap per GPU)",
             "phases_ms": {"insert": float(np.mean(ins_ms)), "deletemin": float(np.mean(del_ms))},
-            "roofline": {"bound": "hbm", "kernel": "bgpq_ops_kernel (DELETEMIN launch)",
+            "roofline": {"bound": "hbm", "kernel": ("bgpq_dtop_kernel (DELETEMIN launch)" if args.mode == "locks" else "bgpq_srv_kernel (DELETEMIN launch)"),
                          "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
                          "traffic": traffic, "peak_source": peak_src,
                          "alg_bytes_per_launch": bm["deletemin"]},
