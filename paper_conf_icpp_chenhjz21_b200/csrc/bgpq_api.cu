@@ -15,6 +15,7 @@
 #include "bgpq_pipe.cuh"
 #include "bgpq_server.cuh"
 #include "bgpq_dtop.cuh"
+#include "bgpq_pipe2.cuh"
 
 using namespace bgpqd;
 
@@ -136,7 +137,19 @@ struct KernelInfo {
   }
   static cudaError_t pipe_launch(int grid, const HeapArgs& H, const PipeArgs& P, const CallArgs& C,
                                  cudaStream_t s) {
-    bgpq_ins_pipe_kernel<K, V, NT><<<grid, NT, pipe_smem_bytes<K, V>(), s>>>(H, P, C);
+    if (g_debug & 32u) {  // test switch: the synchronous pipeline (bgpq_pipe.cuh)
+      bgpq_ins_pipe_kernel<K, V, NT><<<grid, NT, pipe_smem_bytes<K, V>(), s>>>(H, P, C);
+    } else {
+      static bool attr = false;
+      auto kern = bgpq_ins_pipe2_kernel<K, V, NT>;
+      const size_t smem = pipe2_smem_bytes<K, V>();
+      if (!attr) {
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        if (e != cudaSuccess) return e;
+        attr = true;
+      }
+      kern<<<grid, NT + 64, smem, s>>>(H, P, C);
+    }
     g_launches.fetch_add(1);
     return cudaGetLastError();
   }

@@ -8,7 +8,9 @@ dk = torch.from_numpy(keys.view(np.int32)).cuda()
 out = torch.empty(n, dtype=torch.int32, device="cuda")
 q = pkg.BGPQ(capacity=n, K=K, values=False)
 for parts in [int(x) for x in sys.argv[2:]]:
-    q.insert(dk); torch.cuda.synchronize()
+    ei = [torch.cuda.Event(enable_timing=True) for _ in range(2)]
+    ei[0].record(); q.insert(dk); ei[1].record(); torch.cuda.synchronize()
+    print(f"insert ms {ei[0].elapsed_time(ei[1]):.1f}", flush=True)
     e = [torch.cuda.Event(enable_timing=True) for _ in range(parts + 1)]
     step = n // parts
     e[0].record()
