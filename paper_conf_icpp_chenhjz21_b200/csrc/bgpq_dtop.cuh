@@ -64,7 +64,7 @@ struct DtJob {
 // thread-0 state of the top CTA (see dt_top)
 struct DtS {
   u32 fm;  // free slot mask
-  u32 pout;  // slot read by a pending output bulk copy (DT_NONE if none)
+  u32 pout, pout_old;  // slots read by the output bulk copies of this / the previous slot
   u32 wbs, pa0, pb0, pq0, pa1, pb1, pq1;  // write-back sequence, slots pending the helper's read
   u32 hs;
   u32 rs;
@@ -128,7 +128,7 @@ struct DtS {
   u64 tmark;
   __device__ __forceinline__ void init() {
     hs = 0; rs = 0; ps = 0; sph = 0; rph = 0; sbi = 0; rbi = 0; lag_cur = 0; lag_bi = 0; lag_par = 0; lag_s0 = 0; lag_s1 = 0; pre_tar = 0; pre_slot = 0; pre_bi = 0; pre_par = 0; est_y2 = 0; est_bi = 0; est_par = 0; est_s0 = 0; est_s1 = 0; wb0 = 0; wb1 = 0; wb_pub = 0; wb_pending = 0; fr0 = 0; fr1 = 0; fl = 0; size = 0; path = 0; R = 0; remained = 0; rs_old = 0; y1 = 0; y2 = 0; car1 = 0; m1lo = 0; m1hi = 0; mfa = 0; mfb = 0; tsl = 0; lx = 0; ly = 0; lX = 0; lcar = 0; lcar3 = 0; lcf = 0; take_sv = 0; stage = 0; lag = 0; pre = 0; est = 0; walk = 0; walk2 = 0; m1v = 0; conflict = 0; lst = 0; i = 0; nout = 0; tmark = 0;
-    pout = DT_NONE;
+    pout = pout_old = DT_NONE;
     wbs = pq0 = pq1 = 0; pa0 = pb0 = pa1 = pb1 = DT_NONE;
     fr0 = fr1 = car1 = m1lo = m1hi = mfa = mfb = tsl = lX = lcar = lcar3 = lcf = R = DT_NONE;
   }
@@ -173,15 +173,13 @@ __device__ __forceinline__ void grp_bar(int g) {
   asm volatile("bar.sync %0, %1;" ::"r"(2 + g), "n"(DT_GT) : "memory");
 }
 
-// SORT_SPLIT by a group of DT_GT threads (t = index in the group)
+// SORT_SPLIT by a group of DT_GT threads (t = index in the group): warp-cooperative
+// merge path (one ballot co-rank per warp, conflict-free window loads) by default; the
+// per-thread register-window merge path with test switch win (BGPQ_DEBUG bit 64)
 template <int K, bool V>
 __device__ __forceinline__ void grp_split(int t, const u32* zk, const u32* zv, int na, const u32* wk, const u32* wv,
-                                          int nb, int ma, u32* xk, u32* xv, u32* yk, u32* yv) {
-#ifndef BGPQ_DT_WARPMERGE
-#define BGPQ_DT_WARPMERGE 1
-#endif
-  if constexpr (BGPQ_DT_WARPMERGE) {
-    // warp-cooperative merge path: one ballot co-rank per warp, conflict-free window loads
+                                          int nb, int ma, u32* xk, u32* xv, u32* yk, u32* yv, bool win = false) {
+  if (!win) {
     constexpr int NW = (2 * K / 32 < DT_GT / 32) ? 2 * K / 32 : DT_GT / 32;
     grp_merge_warp<K, NW, V>(t >> 5, zk, zv, na, wk, wv, nb, ma, xk, xv, yk, yv);
   } else {
@@ -427,35 +425,39 @@ template <int K, bool V>
 __device__ __forceinline__ bool dt_fast(DTop<K, V>& T, DtS& S) {
   DtCtl* c = T.c;
   const HeapArgs& H = T.H;
-  const u32 fl = S.fl;
-  if (!(fl & F_NEW) || S.path != 3u || S.conflict || !(fl & F_M0) || !S.m1v || S.size != (u32)K ||
-      (S.rs != (u32)K && S.rs != 0u))
+  // ---- the state this path reads, into registers (independent shared-memory loads)
+  const u32 fl = S.fl, path = S.path, conflict = S.conflict, m1v = S.m1v, size = S.size, rs0 = S.rs;
+  const u32 hs0 = S.hs, y1 = S.y1, R = S.R, lo1 = S.m1lo, hi1 = S.m1hi, ps = S.ps;
+  const u64 i = S.i;
+  if (!(fl & F_NEW) || path != 3u || conflict || !(fl & F_M0) || !m1v || size != (u32)K ||
+      (rs0 != (u32)K && rs0 != 0u))
     return false;
+  const bool lag = (fl & F_LAG) != 0;
+  const bool lt = (T.C.debug & 128u) != 0;
+  ull tq = lt ? clock64() : 0;
+#define DT_MARK(k) if (lt) { const ull t_ = clock64(); c->ts[k] += t_ - tq; tq = t_; }
+  const u32 hs = hs0 - 1u;  // after the refill
+  const u32 x1 = y1 ^ 1u, cl = 2u * y1, cr = cl + 1u;
+  if (cr > hs) return false;
   // |root| = 0 (R4: a drained heap keeps heapSize = 1): the whole refilled root is the output
   // (EXTRACT_ROOT(items, remainedSize = K), Alg.3), emitted by one TMA bulk store
-  const bool emit_root = S.rs == 0u;
-  const u64 opos = S.i * (u64)K;
+  const bool emit_root = rs0 == 0u;
+  const u64 opos = i * (u64)K;
   if (emit_root && (((reinterpret_cast<uintptr_t>(T.C.out_k + opos) & 15u) != 0) ||
                     (V && T.C.out_v && (reinterpret_cast<uintptr_t>(T.C.out_v + opos) & 15u) != 0)))
     return false;
-  const bool lag = (fl & F_LAG) != 0;
-  const u32 hs = S.hs - 1u;  // after the refill
-  // ---- loads (independent)
-  const u32 y1 = S.y1, x1 = y1 ^ 1u, cl = 2u * y1, cr = cl + 1u;
-  if (cr > hs) return false;
-  const u32 R = S.R, nl = c->ns[cl], nr = c->ns[cr], n2 = c->ns[2], n3 = c->ns[3];
-  const u32 lo0 = c->p_m[0][2], hi0 = c->p_m[0][3], lo1 = S.m1lo, hi1 = S.m1hi;
+  const u32 nl = c->ns[cl], nr = c->ns[cr], n2 = c->ns[2], n3 = c->ns[3], oroot = c->ns[1];
+  const u32 lo0 = c->p_m[0][2], hi0 = c->p_m[0][3];
   const u32 Rmax = T.kmax(R), Rmin = T.kmin(R);
   const u32 min2 = T.kmin(n2), min3 = T.kmin(n3), max2 = T.kmax(n2);
   const u32 lo0max = T.kmax(lo0), lo1max = T.kmax(lo1);
   const u32 minl = T.kmin(nl), minr = T.kmin(nr), maxl = T.kmax(nl), maxr = T.kmax(nr);
-  const u32 ps = S.ps;
   const u32 pbmin = ps ? T.kmin(c->ns[0]) : KEY_MAX;
   u32 lcur = 0, lcar = DT_NONE, lo2 = DT_NONE, hi2 = DT_NONE, st0 = 0, st1 = 0, mn0 = 0, mn1 = 0, mx0 = 0, mx1 = 0;
-  u32 lcarmax = 0, lcarmin = 0, lo2max = 0;
+  u32 lcarmax = 0, lcarmin = 0, lo2max = 0, lag_s0 = 0, lag_s1 = 0;
   if (lag) {
     const u32 bi = S.lag_bi;
-    lcur = S.lag_cur;
+    lcur = S.lag_cur; lag_s0 = S.lag_s0; lag_s1 = S.lag_s1;
     lcar = c->ns[lcur];
     lo2 = c->p_m[2][2]; hi2 = c->p_m[2][3];
     st0 = c->stg_st[bi][0]; st1 = c->stg_st[bi][1];
@@ -474,31 +476,37 @@ __device__ __forceinline__ bool dt_fast(DTop<K, V>& T, DtS& S) {
     if (lcarmax <= min(mn0, mn1)) return false;                 // l.4 stop at y2(i-1)
     if (lo2max > lcarmin) return false;                         // l.12 not a swap at y2(i-1)
   }
-  // ---- commit: op i-1's depth-2 step
-  ull* st = c->st;
+  DT_MARK(0)
+  u32 fm = S.fm;
+  u32 d_lv = 2, d_merge = 0, d_nomove = 0;
+  // ---- commit: op i-1's depth-2 step (l.9-12), write-back + hand-over by helper B
   if (lag) {
     const u32 c0 = 2u * lcur, c1 = c0 + 1u;
     const u32 x3 = mx0 > mx1 ? c0 : c1, y3 = mx0 > mx1 ? c1 : c0;  // l.9 (R6)
-    st[S_DEL_LEVELS]++;
-    st[(mx0 <= mn1) ? S_DEL_LR_NOMOVE : S_DEL_LR_MERGE]++;
-    st[S_DEL_CY_SWAP]++;
+    ++d_lv;
+    if (mx0 <= mn1) ++d_nomove; else ++d_merge;
     c->ns[lcur] = lo2;
-    T.release_slot(S, S.lag_s0); T.release_slot(S, S.lag_s1);
-    T.writeback(S, x3, hi2, y3, lcar, 2u * y3 <= S.hs);  // a walker continues at y3 (l.15)
+    fm |= (1u << lag_s0) | (1u << lag_s1);
+    const u32 seq = S.wbs + 1u;
+    S.wbs = seq;
+    T.enqueue(RQ_WB2, x3, hi2, y3, lcar, ((2u * y3 <= hs0) ? 1u : 0u) | (seq << 1), T.kmin(hi2), T.kmax(hi2),
+              lcarmin, lcarmax);
+    // slots of the write-back two generations ago: free once helper B has read them
+    const u32 pq1 = S.pq1;
+    if (pq1 != 0) {
+      while ((int)(*reinterpret_cast<volatile u32*>(&c->wb_rd) - pq1) < 0) __nanosleep(32);
+      fm |= (1u << S.pa1) | (1u << S.pb1);
+    }
+    S.pa1 = S.pa0; S.pb1 = S.pb0; S.pq1 = S.pq0;
+    S.pa0 = hi2; S.pb0 = lcar; S.pq0 = seq;
     S.lag = 0;
   }
+  DT_MARK(1)
   // ---- commit: op i (Alg.2 refill path, Alg.3 at the root and at y1)
-  st[S_DEL_OPS]++;
-  st[S_DEL_REFILL]++;
-  st[S_DEL_LEVELS] += 2;
-  st[(max2 <= min3) ? S_DEL_LR_NOMOVE : S_DEL_LR_MERGE]++;
-  st[(maxl <= minr) ? S_DEL_LR_NOMOVE : S_DEL_LR_MERGE]++;
-  st[S_DEL_CY_SWAP] += 2;
-  S.nout += (u32)K;
-  S.hs = hs;
-  T.release_slot(S, c->ns[1]);  // old root (output in phase A)
-  T.release_slot(S, n2); T.release_slot(S, n3);
-  T.release_slot(S, nl); T.release_slot(S, nr);
+  if (max2 <= min3) ++d_nomove; else ++d_merge;
+  if (maxl <= minr) ++d_nomove; else ++d_merge;
+  S.pout = oroot;  // old root: read by phase A's output copy, freed after its bulk read
+  fm |= (1u << n2) | (1u << n3) | (1u << nl) | (1u << nr);
   c->ns[1] = lo0;
   c->ns[x1] = hi0;
   if (emit_root) {
@@ -517,29 +525,180 @@ __device__ __forceinline__ bool dt_fast(DTop<K, V>& T, DtS& S) {
   c->ns[x2] = hi1;
   c->ns[y2] = R;
   S.m1v = 0;
+  S.nout += (u32)K;
+  S.hs = hs;
   // op i's depth-2 step goes to the next slot
-  if (S.est && !(2u * y2 <= hs && S.est_y2 == y2)) {  // (not expected: the prediction is exact)
-    T.enqueue(RQ_WB, 2u * S.est_y2, 2u * S.est_y2 + 1u <= H.cap ? 2u * S.est_y2 + 1u : 0u, 0u);
+  u32 est = S.est;
+  const u32 est_y2 = S.est_y2;
+  if (est && !(2u * y2 <= hs && est_y2 == y2)) {  // (not expected: the prediction is exact)
+    T.enqueue(RQ_WB, 2u * est_y2, 2u * est_y2 + 1u <= H.cap ? 2u * est_y2 + 1u : 0u, 0u);
     mbar_wait(&c->sbar[S.est_bi], S.est_par);
-    T.release_slot(S, S.est_s0); T.release_slot(S, S.est_s1);
-    S.est = 0;
+    fm |= (1u << S.est_s0) | (1u << S.est_s1);
+    est = 0;
   }
   if (2u * y2 <= hs) {
     S.lag = 1; S.lag_cur = y2;
-    if (S.est) {
+    if (est) {
       S.lag_bi = S.est_bi; S.lag_par = S.est_par; S.lag_s0 = S.est_s0; S.lag_s1 = S.est_s1;
-      S.est = 0;
+      est = 0;
     } else {
       const u32 c0 = 2u * y2, c1 = c0 + 1u;
-      S.lag_s0 = T.alloc(S); S.lag_s1 = T.alloc(S);
-      S.lag_bi = S.sbi; S.lag_par = (S.sph >> S.sbi) & 1u;
-      T.enqueue(RQ_STAGE, c0, c1 <= H.cap ? c1 : 0u, S.lag_s0, S.lag_s1, S.sbi);
-      S.sph ^= 1u << S.sbi; S.sbi ^= 1u;
+      if (fm == 0) __trap();
+      const u32 sa = __ffs(fm) - 1; fm &= ~(1u << sa);
+      if (fm == 0) __trap();
+      const u32 sb = __ffs(fm) - 1; fm &= ~(1u << sb);
+      const u32 sbi = S.sbi, sph = S.sph;
+      S.lag_s0 = sa; S.lag_s1 = sb;
+      S.lag_bi = sbi; S.lag_par = (sph >> sbi) & 1u;
+      T.enqueue(RQ_STAGE, c0, c1 <= H.cap ? c1 : 0u, sa, sb, sbi);
+      S.sph = sph ^ (1u << sbi); S.sbi = sbi ^ 1u;
     }
   }
-  S.i += 1;
+  S.est = est;
+  S.fm = fm;
+  S.i = i + 1;
   S.stage = 99;
+  // device counters (byte model)
+  ull* st = c->st;
+  st[S_DEL_OPS] += 1;
+  st[S_DEL_REFILL] += 1;
+  st[S_DEL_LEVELS] += d_lv;
+  st[S_DEL_LR_MERGE] += d_merge;
+  st[S_DEL_LR_NOMOVE] += d_nomove;
+  st[S_DEL_CY_SWAP] += d_lv;
+  DT_MARK(2)
   return true;
+}
+
+// Plan of the next slot (thread 0): which operation runs, its refill source, the splits the
+// three groups run in phase A, and the helper requests that can be issued ahead (refill node
+// of op i+1, depth-3 children of op i).  The state it touches is loaded into registers once
+// and written back once (shared-memory round trips serialise single-thread code).
+template <int K, bool V>
+__device__ __forceinline__ void dt_plan(DTop<K, V>& T, DtS& S, const u64 n_ops, const bool timing) {
+  DtCtl* c = T.c;
+  const HeapArgs& H = T.H;
+  const CallArgs& C = T.C;
+  const bool lt = (C.debug & 128u) != 0;
+  ull tq = lt ? clock64() : 0;
+  const ull twg = timing ? clock64() : 0;
+  // output copies (one bulk group per slot, issued by this thread): all but the newest have
+  // read their source slot, which is freed now; the newest one's slot is freed next slot
+  asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
+  if (timing) c->ts[10] += clock64() - twg;
+  u32 fm = S.fm;
+  if (S.pout_old != DT_NONE) fm |= 1u << S.pout_old;
+  S.pout_old = S.pout;
+  S.pout = DT_NONE;
+  auto alloc = [&]() -> u32 {
+    if (fm == 0) __trap();  // slot budget exceeded: a bug, never silent corruption
+    const u32 q = __ffs(fm) - 1;
+    fm &= ~(1u << q);
+    return q;
+  };
+  const u64 i = S.i;
+  const u32 hs = S.hs, rs = S.rs, lag = S.lag, lag_cur = S.lag_cur;
+  u32 pre = S.pre;
+  const u32 pre_tar = S.pre_tar;
+  u32 rbi = S.rbi, rph = S.rph, sbi = S.sbi, sph = S.sph;
+  if (C.prog) { C.prog[0] = (u32)i; C.prog[1] = 1; C.prog[4] = hs; C.prog[5] = lag ? (0x80000000u | lag_cur) : 0u; C.prog[6] = pre ? pre_tar : 0u; }
+  u32 fl = 0;
+  bool new_op = i < n_ops;
+  const bool pipelined = pre && pre_tar == hs;
+  if (new_op && lag && !pipelined) new_op = false;  // small heap: finish op i-1 first
+  if (!new_op && !lag) {
+    c->p_flags = DT_NONE;
+    S.fm = fm;
+    return;
+  }
+  if (lag) {
+    fl |= F_LAG;
+    c->p_m[2][0] = S.lag_s0; c->p_m[2][1] = S.lag_s1;
+    c->p_m[2][2] = alloc(); c->p_m[2][3] = alloc();
+    c->p_sbi = S.lag_bi; c->p_spar = S.lag_par;
+  }
+  u32 rwait = 0, conflict = 0, m1v = 0, y1 = 0;
+  if (new_op) {
+    fl |= F_NEW;
+    const u64 rem = C.n - i * (u64)K;
+    const u32 size = (u32)(rem < (u64)K ? rem : (u64)K);
+    const u32 path = hs == 0 ? 0u : size < rs ? 1u : hs == 1 ? 2u : 3u;  // EMPTY EXTRACT PBUF REFILL
+    S.size = size; S.path = path; S.rs_old = rs;
+    c->p_out_slot = c->ns[1];
+    c->p_out_n = path == 1 ? size : (path >= 2 ? rs : 0u);
+    c->p_iop_lo = (u32)i; c->p_iop_hi = (u32)(i >> 32);
+    if (path == 3) {
+      const u32 hn = hs - 1u;
+      u32 R;
+      if (pipelined) {  // Alg.2 l.6-12 done ahead by the helper
+        R = S.pre_slot;
+        rwait = 1; c->p_rbi = S.pre_bi; c->p_rpar = S.pre_par;
+        pre = 0;
+      } else if (hs <= 7u) {  // the last node is on chip
+        R = c->ns[hs];
+        c->ns[hs] = DT_NONE;
+      } else {  // synchronous take by the helper
+        R = alloc();
+        T.enqueue(RQ_REFILL, hs, R, rbi);
+        rwait = 1; c->p_rbi = rbi; c->p_rpar = (rph >> rbi) & 1u;
+        rph ^= 1u << rbi; rbi ^= 1u;
+      }
+      S.R = R;
+      // op i's path and its speculative l/r splits (l.9-10 on cached max keys)
+      const bool a2 = 2u <= hn, a3 = 3u <= hn;
+      const u32 n2 = c->ns[2], n3 = c->ns[3];
+      if (a2 && a3) {
+        fl |= F_M0;
+        c->p_m[0][0] = n2; c->p_m[0][1] = n3;
+        c->p_m[0][2] = alloc(); c->p_m[0][3] = alloc();
+        y1 = T.kmax(n2) > T.kmax(n3) ? 3u : 2u;  // R6: tie -> x = r, y = l
+      } else if (a2) {
+        y1 = 2u;
+      }
+      DT_MARK(3)
+      // take the refill node of op i+1 ahead (deep node, full-K op)
+      if (i + 1 < n_ops && C.n - (i + 1) * (u64)K >= (u64)K && hn >= DT_BIG) {
+        const u32 ps_ = alloc();
+        pre = 1; S.pre_tar = hn; S.pre_slot = ps_;
+        S.pre_bi = rbi; S.pre_par = (rph >> rbi) & 1u;
+        T.enqueue(RQ_REFILL, hn, ps_, rbi);
+        rph ^= 1u << rbi; rbi ^= 1u;
+      }
+      DT_MARK(4)
+      if (y1) {
+        const u32 cl = 2u * y1, cr = cl + 1u;
+        const bool al = cl <= hn, ar = cr <= hn;
+        const u32 ncl = c->ns[cl], ncr = c->ns[cr];
+        conflict = lag && (lag_cur == cl || lag_cur == cr);
+        if (al && ar && !conflict) {
+          fl |= F_M1;
+          m1v = 1;
+          const u32 lo = alloc(), hi = alloc();
+          S.m1lo = lo; S.m1hi = hi;
+          c->p_m[1][0] = ncl; c->p_m[1][1] = ncr;
+          c->p_m[1][2] = lo; c->p_m[1][3] = hi;
+        }
+        if (pipelined && !conflict && (al || ar)) {  // lock + stage op i's depth-3 children now
+          const u32 p2 = (al && ar) ? (T.kmax(ncl) > T.kmax(ncr) ? cr : cl) : (al ? cl : cr);
+          const u32 c0 = 2u * p2, c1 = c0 + 1u;
+          if (c0 <= hn) {
+            const u32 e0 = alloc(), e1 = alloc();
+            S.est = 1; S.est_y2 = p2; S.est_s0 = e0; S.est_s1 = e1;
+            S.est_bi = sbi; S.est_par = (sph >> sbi) & 1u;
+            T.enqueue(RQ_STAGE, c0, c1 <= H.cap ? c1 : 0u, e0, e1, sbi);
+            sph ^= 1u << sbi; sbi ^= 1u;
+          }
+        }
+      }
+      DT_MARK(5)
+    }
+  }
+  c->p_rwait = rwait;
+  c->p_flags = fl;
+  S.fl = fl; S.m1v = m1v; S.conflict = conflict; S.walk = 0; S.walk2 = 0; S.y1 = y1;
+  S.pre = pre; S.rbi = rbi; S.rph = rph; S.sbi = sbi; S.sph = sph;
+  S.fm = fm;
+  DT_MARK(6)
 }
 
 template <int K, bool V>
@@ -581,109 +740,18 @@ __device__ __forceinline__ void dt_top(DTop<K, V>& T) {
   cta_bar<DT_NTC>();
 
   const bool timing = (C.debug & 8u) != 0;
+  const bool ltime = timing || (C.debug & 128u) != 0;  // light timing: plan / phase A / phase B only
+  const bool mwin = (C.debug & 64u) != 0;
+  // the first plan; every later one is made by thread 0 at the end of the previous slot's
+  // phase B, so a common slot has two CTA barriers (after phase A, after phase B)
+  if (tid == 0 && ltime) SS.tmark = clock64();
+  if (tid == 0) dt_plan<K, V>(T, SS, n_ops, timing);
+  cta_bar<DT_NTC>();
   for (;;) {
-    // =========================== plan (thread 0) ===========================
-    if (tid == 0 && timing) SS.tmark = clock64();
-    if (tid == 0) {
-      DtS* __restrict__ const Sp = &SS;
-      DtS& S = *Sp;
-      const ull twg = timing ? clock64() : 0;
-      asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");  // the last output copy has read its slot
-      if (timing) c->ts[10] += clock64() - twg;
-      T.release_slot(S, S.pout);
-      S.pout = DT_NONE;
-      if (C.prog) { C.prog[0] = (u32)S.i; C.prog[1] = 1; C.prog[4] = S.hs; C.prog[5] = S.lag ? (0x80000000u | S.lag_cur) : 0u; C.prog[6] = S.pre ? S.pre_tar : 0u; }
-      S.fl = 0;
-      bool new_op = S.i < n_ops;
-      const bool pipelined = S.pre && S.pre_tar == S.hs;
-      if (new_op && S.lag && !pipelined) new_op = false;  // small heap: finish op i-1 first
-      if (!new_op && !S.lag) {
-        c->p_flags = DT_NONE;
-      } else {
-        if (S.lag) {
-          S.fl |= F_LAG;
-          c->p_m[2][0] = S.lag_s0; c->p_m[2][1] = S.lag_s1;
-          c->p_m[2][2] = T.alloc(S); c->p_m[2][3] = T.alloc(S);
-          c->p_sbi = S.lag_bi; c->p_spar = S.lag_par;
-        }
-        c->p_rwait = 0;
-        S.m1v = false; S.conflict = false; S.walk = S.walk2 = false;
-        if (new_op) {
-          S.fl |= F_NEW;
-          const u64 rem = C.n - S.i * (u64)K;
-          S.size = (u32)(rem < (u64)K ? rem : (u64)K);
-          S.path = S.hs == 0 ? 0u : S.size < S.rs ? 1u : S.hs == 1 ? 2u : 3u;  // EMPTY EXTRACT PBUF REFILL
-          c->p_out_slot = c->ns[1];
-          c->p_out_n = S.path == 1 ? S.size : (S.path >= 2 ? S.rs : 0u);
-          c->p_iop_lo = (u32)S.i; c->p_iop_hi = (u32)(S.i >> 32);
-          S.rs_old = S.rs;
-          if (S.path == 3) {
-            const u32 hn = S.hs - 1u;
-            if (pipelined) {  // Alg.2 l.6-12 done ahead by the helper
-              S.R = S.pre_slot;
-              c->p_rwait = 1; c->p_rbi = S.pre_bi; c->p_rpar = S.pre_par;
-              S.pre = false;
-            } else if (S.hs <= 7u) {  // the last node is on chip
-              S.R = c->ns[S.hs];
-              c->ns[S.hs] = DT_NONE;
-            } else {  // synchronous take by the helper
-              S.R = T.alloc(S);
-              T.enqueue(RQ_REFILL, S.hs, S.R, S.rbi);
-              c->p_rwait = 1; c->p_rbi = S.rbi; c->p_rpar = (S.rph >> S.rbi) & 1u;
-              S.rph ^= 1u << S.rbi; S.rbi ^= 1u;
-            }
-            // op i's path and its speculative l/r splits (l.9-10 on cached max keys)
-            const bool a2 = 2u <= hn, a3 = 3u <= hn;
-            S.y1 = 0;
-            if (a2 && a3) {
-              S.fl |= F_M0;
-              c->p_m[0][0] = c->ns[2]; c->p_m[0][1] = c->ns[3];
-              c->p_m[0][2] = T.alloc(S); c->p_m[0][3] = T.alloc(S);
-              S.y1 = T.kmax(c->ns[2]) > T.kmax(c->ns[3]) ? 3u : 2u;  // R6: tie -> x = r, y = l
-            } else if (a2) {
-              S.y1 = 2u;
-            }
-            // take the refill node of op i+1 ahead (deep node, full-K op)
-            if (S.i + 1 < n_ops && C.n - (S.i + 1) * (u64)K >= (u64)K && hn >= DT_BIG) {
-              S.pre = true; S.pre_tar = hn; S.pre_slot = T.alloc(S);
-              S.pre_bi = S.rbi; S.pre_par = (S.rph >> S.rbi) & 1u;
-              T.enqueue(RQ_REFILL, hn, S.pre_slot, S.rbi);
-              S.rph ^= 1u << S.rbi; S.rbi ^= 1u;
-            }
-            if (S.y1) {
-              const u32 cl = 2u * S.y1, cr = cl + 1u;
-              const bool al = cl <= hn, ar = cr <= hn;
-              S.conflict = S.lag && (S.lag_cur == cl || S.lag_cur == cr);
-              if (al && ar && !S.conflict) {
-                S.fl |= F_M1;
-                S.m1v = true;
-                S.m1lo = T.alloc(S); S.m1hi = T.alloc(S);
-                c->p_m[1][0] = c->ns[cl]; c->p_m[1][1] = c->ns[cr];
-                c->p_m[1][2] = S.m1lo; c->p_m[1][3] = S.m1hi;
-              }
-              if (pipelined && !S.conflict && (al || ar)) {  // lock + stage op i's depth-3 children now
-                const u32 p2 = (al && ar) ? (T.kmax(c->ns[cl]) > T.kmax(c->ns[cr]) ? cr : cl) : (al ? cl : cr);
-                const u32 c0 = 2u * p2, c1 = c0 + 1u;
-                if (c0 <= hn) {
-                  S.est = true; S.est_y2 = p2;
-                  S.est_s0 = T.alloc(S); S.est_s1 = T.alloc(S);
-                  S.est_bi = S.sbi; S.est_par = (S.sph >> S.sbi) & 1u;
-                  T.enqueue(RQ_STAGE, c0, c1 <= H.cap ? c1 : 0u, S.est_s0, S.est_s1, S.sbi);
-                  S.sph ^= 1u << S.sbi; S.sbi ^= 1u;
-                }
-              }
-            }
-          }
-        }
-        c->p_flags = S.fl;
-      }
-      (void)0;
-    }
-    cta_bar<DT_NTC>();
     const u32 pf = c->p_flags;
     if (pf == DT_NONE) break;
     if (tid == 0 && C.prog) C.prog[1] = 2;
-    if (tid == 0 && timing) { const ull t = clock64(); c->tm[0] += t - SS.tmark; SS.tmark = t; c->tm[5]++; if (SS.conflict) c->tm[6]++; }
+    if (tid == 0 && ltime) { const ull t = clock64(); c->tm[0] += t - SS.tmark; SS.tmark = t; c->tm[5]++; if (SS.conflict) c->tm[6]++; }
 
     // =========================== phase A: concurrent work ===========================
     const ull tg0 = (timing && gt == 0) ? clock64() : 0;
@@ -718,13 +786,13 @@ __device__ __forceinline__ void dt_top(DTop<K, V>& T) {
       if (pf & F_M0) {
         const u32* m = c->p_m[0];
         grp_split<K, V>(gt, T.BK(m[0]), T.BV(m[0]), K, T.BK(m[1]), T.BV(m[1]), K, K, T.BK(m[2]), T.BV(m[2]),
-                        T.BK(m[3]), T.BV(m[3]));
+                        T.BK(m[3]), T.BV(m[3]), mwin);
       }
     } else if (g == 1) {
       if (pf & F_M1) {
         const u32* m = c->p_m[1];
         grp_split<K, V>(gt, T.BK(m[0]), T.BV(m[0]), K, T.BK(m[1]), T.BV(m[1]), K, K, T.BK(m[2]), T.BV(m[2]),
-                        T.BK(m[3]), T.BV(m[3]));
+                        T.BK(m[3]), T.BV(m[3]), mwin);
       }
     } else {
       if (pf & F_LAG) {
@@ -735,16 +803,18 @@ __device__ __forceinline__ void dt_top(DTop<K, V>& T) {
         if (c->stg_st[bi][0] == ST_AVAIL && c->stg_st[bi][1] == ST_AVAIL) {
           const u32* m = c->p_m[2];
           grp_split<K, V>(gt, T.BK(m[0]), T.BV(m[0]), K, T.BK(m[1]), T.BV(m[1]), K, K, T.BK(m[2]), T.BV(m[2]),
-                          T.BK(m[3]), T.BV(m[3]));
+                          T.BK(m[3]), T.BV(m[3]), mwin);
         }
       }
     }
     if (timing && gt == 0) c->tm[8 + g] += clock64() - tg0;
     cta_bar<DT_NTC>();
-    if (tid == 0 && timing) { const ull t = clock64(); c->tm[1] += t - SS.tmark; SS.tmark = t; }
+    if (tid == 0 && ltime) { const ull t = clock64(); c->tm[1] += t - SS.tmark; SS.tmark = t; }
     // every thread observes the TMA data phase B may read
+    const ull tw7 = (tid == 0 && ltime) ? clock64() : 0;
     if (pf & F_LAG) mbar_wait(&c->sbar[c->p_sbi], c->p_spar);
     if (c->p_rwait) mbar_wait(&c->rbar[c->p_rbi], c->p_rpar);
+    if (tid == 0 && ltime) c->ts[7] += clock64() - tw7;
     if (tid == 0 && timing) { const ull t = clock64(); c->tm[3] += t - SS.tmark; SS.tmark = t; }
 
     // =========================== phase B: decisions + job rounds ===========================
@@ -853,6 +923,7 @@ __device__ __forceinline__ void dt_top(DTop<K, V>& T) {
                 S.remained = S.size - S.rs;
                 S.nout += S.size;
                 S.hs -= 1u;
+                asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
                 T.release_slot(S, c->ns[1]);  // the old root, output in phase A
                 c->ns[1] = DT_NONE;
                 S.mfa = S.mfb = DT_NONE;
@@ -867,6 +938,7 @@ __device__ __forceinline__ void dt_top(DTop<K, V>& T) {
               break;
             }
             case 30: {
+              asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");  // phase A output read it
               T.release_slot(S, c->ns[1]);
               c->ns[1] = S.tsl;
               S.rs -= S.size;
@@ -875,6 +947,7 @@ __device__ __forceinline__ void dt_top(DTop<K, V>& T) {
             }
             case 31: {
               const u32 take = S.take_sv;
+              asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");  // phase A output read it
               T.release_slot(S, c->ns[1]);
               T.release_slot(S, c->ns[0]);
               c->ns[0] = DT_NONE;
@@ -1019,6 +1092,10 @@ __device__ __forceinline__ void dt_top(DTop<K, V>& T) {
           }
           if (timing) c->ts[st_in >= 30 ? 8 : (st_in > 8 ? 8 : st_in)] += clock64() - tsw;
         }
+        if (done) {  // the slot is complete: plan the next one now
+          if (ltime) { const ull t = clock64(); c->tm[4] += t - SS.tmark; SS.tmark = t; }
+          dt_plan<K, V>(T, SS, n_ops, timing);
+        }
         c->more = done ? 0u : 1u;
         if (C.prog) C.prog[1] = 100 + S.stage;
         (void)0;
@@ -1028,11 +1105,10 @@ __device__ __forceinline__ void dt_top(DTop<K, V>& T) {
       cta_bar<DT_NTC>();
       T.run_jobs();
       const u32 more = c->more;
+      if (!more) break;  // no job list follows: thread 0 writes none before the next phase A
       cta_bar<DT_NTC>();
       if (tid == 0 && timing) c->ts[11] += clock64() - trd;
-      if (!more) break;
     }
-    if (tid == 0 && timing) c->tm[4] += clock64() - SS.tmark;
   }
 
   // =========================== call end: write the on-chip part back ===========================
@@ -1073,7 +1149,7 @@ __device__ __forceinline__ void dt_top(DTop<K, V>& T) {
     ull* stat = reinterpret_cast<ull*>(H.hdr + H_STAT);
     for (int q = 0; q < NSTAT; ++q)
       if (c->st[q]) atomicAdd(stat + q, c->st[q]);
-    if (timing) {
+    if (ltime) {
       ull* tms = reinterpret_cast<ull*>(H.hdr + H_TIME);
       for (int q = 0; q < 12; ++q) { atomicAdd(tms + 16 + q, c->tm[q]); atomicAdd(tms + q, c->ts[q]); }
     }

@@ -24,5 +24,5 @@ for i, nm in enumerate(["plan", "phaseA", "G2 stage wait", "refill wait", "phase
     print("  %-14s %8.0f cyc/slot" % (nm, d[16 + i] / slots))
 print("  helper lock wait %8.0f cyc/slot" % (d[23] / slots))
 print("  G0 out+merge %8.0f  G1 merge %8.0f  G2 wait+merge %8.0f  rounds/slot %.2f" % (d[24] / slots, d[25] / slots, d[26] / slots, d[27] / slots))
-print("  stage cycles/slot:", {nm: round(d[k] / slots) for k, nm in enumerate(["lag1", "lag2", "defer", "root", "step0", "extract", "step1", "st7", "st8+", "enqueue(all)", "plan_waitgroup", "rounds"])})
+print("  stage cycles/slot:", {nm: round(d[k] / slots) for k, nm in enumerate(["fast:loads+tests", "fast:lag commit", "fast:rest", "plan:to refill", "plan:refill enq", "plan:m1+stage enq", "plan:writeback", "B waits", "-", "-", "-", "-"])})
 print("sorted", bool(np.array_equal(out.cpu().numpy().view(np.uint32), np.sort(keys))))
