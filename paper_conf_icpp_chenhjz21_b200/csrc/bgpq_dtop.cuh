@@ -64,6 +64,9 @@ struct DtJob {
 // thread-0 state of the top CTA (see dt_top)
 struct DtS {
   u32 fm;  // free slot mask
+  u32 eseq;              // early-split sequence number
+  u32 est_lo, est_hi;    // output slots of the early depth-2 split of the staged children (G2, phase B)
+  u32 lag_early, lag_lo, lag_hi;  // the pending lag step's split was done early into lag_lo / lag_hi
   u32 pout, pout_old;  // slots read by the output bulk copies of this / the previous slot
   u32 wbs, pa0, pb0, pq0, pa1, pb1, pq1;  // write-back sequence, slots pending the helper's read
   u32 hs;
@@ -129,6 +132,7 @@ struct DtS {
   __device__ __forceinline__ void init() {
     hs = 0; rs = 0; ps = 0; sph = 0; rph = 0; sbi = 0; rbi = 0; lag_cur = 0; lag_bi = 0; lag_par = 0; lag_s0 = 0; lag_s1 = 0; pre_tar = 0; pre_slot = 0; pre_bi = 0; pre_par = 0; est_y2 = 0; est_bi = 0; est_par = 0; est_s0 = 0; est_s1 = 0; wb0 = 0; wb1 = 0; wb_pub = 0; wb_pending = 0; fr0 = 0; fr1 = 0; fl = 0; size = 0; path = 0; R = 0; remained = 0; rs_old = 0; y1 = 0; y2 = 0; car1 = 0; m1lo = 0; m1hi = 0; mfa = 0; mfb = 0; tsl = 0; lx = 0; ly = 0; lX = 0; lcar = 0; lcar3 = 0; lcf = 0; take_sv = 0; stage = 0; lag = 0; pre = 0; est = 0; walk = 0; walk2 = 0; m1v = 0; conflict = 0; lst = 0; i = 0; nout = 0; tmark = 0;
     pout = pout_old = DT_NONE;
+    est_lo = est_hi = lag_lo = lag_hi = DT_NONE; lag_early = 0;
     wbs = pq0 = pq1 = 0; pa0 = pb0 = pa1 = pb1 = DT_NONE;
     fr0 = fr1 = car1 = m1lo = m1hi = mfa = mfb = tsl = lX = lcar = lcar3 = lcf = R = DT_NONE;
   }
@@ -141,6 +145,7 @@ struct DtCtl {
   u32 rq_head[2];  // thread 0 -> helper A (ring 0: STAGE, REFILL) / helper B (ring 1: WB, WB2)
   u32 rq_done[2];  // helper progress
   u32 rq[2][DT_RQ][10];
+  u64 qbar[2][DT_RQ];  // entry h of ring r is published by an arrive on qbar[r][h % DT_RQ]
   u32 wb_rd;     // helper: sequence number of the last RQ_WB2 whose smem slots were read
   u32 stg_st[2][2], stg_min[2][2], stg_max[2][2];
   u32 tasks;     // tasks published (helper)
@@ -151,6 +156,8 @@ struct DtCtl {
   u32 p_out_slot, p_out_n, p_iop_lo, p_iop_hi;
   u32 p_m[3][4]; // group g: split slots z, w -> lo, hi
   u32 p_sbi, p_spar, p_rwait, p_rbi, p_rpar;
+  u32 g2_done;   // G2: sequence number of the last early split finished
+  u32 p_e[7];    // early depth-2 split for G2 in phase B: staged s0, s1 -> lo, hi; sbar index, parity
   u32 more;      // another job round follows
   u32 njobs;
   DtJob job[12];
@@ -159,7 +166,7 @@ struct DtCtl {
   ull ts[12];    // debug: thread-0 cycles per phase-B stage
   ull tm[12];    // debug timers (C.debug & 8): plan, phase A, G2 stage wait, refill wait, phase B, slots, conflicts, helper lock wait
 };
-enum : u32 { F_NEW = 1, F_LAG = 2, F_M0 = 4, F_M1 = 8 };
+enum : u32 { F_NEW = 1, F_LAG = 2, F_M0 = 4, F_M1 = 8, F_LAGDONE = 16, F_EARLY = 32 };
 constexpr size_t DTCTL_BYTES = (sizeof(DtCtl) + 127) / 128 * 128;
 
 template <int K, bool V>
@@ -226,12 +233,16 @@ struct DTop {
     const ull tq = (C.debug & 8u) ? clock64() : 0;
     const u32 r = (type == RQ_STAGE || type == RQ_REFILL) ? 0u : 1u;
     const u32 h = c->rq_head[r];
-    while (h - *reinterpret_cast<volatile u32*>(&c->rq_done[r]) >= (u32)DT_RQ) __nanosleep(32);
-    (void)ld_acq_cta(&c->rq_done[r]);
+    if (h - *reinterpret_cast<volatile u32*>(&c->rq_done[r]) >= (u32)DT_RQ) {
+      while (h - *reinterpret_cast<volatile u32*>(&c->rq_done[r]) >= (u32)DT_RQ) __nanosleep(32);
+      (void)ld_acq_cta(&c->rq_done[r]);
+    }
     u32* e = c->rq[r][h % DT_RQ];
     e[0] = type; e[1] = a0; e[2] = a1; e[3] = a2; e[4] = a3; e[5] = a4;
     e[6] = a5; e[7] = a6; e[8] = a7; e[9] = a8;
-    st_rel_cta(&c->rq_head[r], h + 1u);
+    c->rq_head[r] = h + 1u;  // (thread 0's own counter)
+    // publish: mbarrier arrive (release, CTA scope); the helper's try_wait acquires
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_addr(&c->qbar[r][h % DT_RQ])) : "memory");
     if (C.debug & 8u) c->ts[9] += clock64() - tq;
   }
   // ---- thread 0: hand the write-back of a lag step to the helper (RQ_WB2): node x <- slot X
@@ -303,10 +314,12 @@ __device__ __forceinline__ void dt_helper(DTop<K, V>& T, const u32 hr) {
   const u32 NB = K * 4u;
   u32 seen = 0;
   for (;;) {
-    u32 h;
-    while ((h = *reinterpret_cast<volatile u32*>(&c->rq_head[hr])) == seen) __nanosleep(32);
-    h = ld_acq_cta(&c->rq_head[hr]);
-    while (seen != h) {
+    {
+      u64* qb = &c->qbar[hr][seen % DT_RQ];
+      const u32 par = (seen / DT_RQ) & 1u;
+      while (!mbar_test(qb, par)) __nanosleep(20);
+    }
+    {
       const u32* e = c->rq[hr][seen % DT_RQ];
       const u32 type = e[0];
       if (T.C.prog) { T.C.prog[2 + 5 * hr] = seen; T.C.prog[3 + 5 * hr] = (type << 24) | (e[1] & 0xFFFFFFu); }
@@ -533,13 +546,18 @@ __device__ __forceinline__ bool dt_fast(DTop<K, V>& T, DtS& S) {
   if (est && !(2u * y2 <= hs && est_y2 == y2)) {  // (not expected: the prediction is exact)
     T.enqueue(RQ_WB, 2u * est_y2, 2u * est_y2 + 1u <= H.cap ? 2u * est_y2 + 1u : 0u, 0u);
     mbar_wait(&c->sbar[S.est_bi], S.est_par);
+    if (S.est_lo != DT_NONE)
+      while (*reinterpret_cast<volatile u32*>(&c->g2_done) != S.eseq) __nanosleep(32);  // G2's early split
     fm |= (1u << S.est_s0) | (1u << S.est_s1);
+    if (S.est_lo != DT_NONE) fm |= (1u << S.est_lo) | (1u << S.est_hi);
     est = 0;
   }
+  S.lag_early = 0;
   if (2u * y2 <= hs) {
     S.lag = 1; S.lag_cur = y2;
     if (est) {
       S.lag_bi = S.est_bi; S.lag_par = S.est_par; S.lag_s0 = S.est_s0; S.lag_s1 = S.est_s1;
+      S.lag_early = S.est_lo != DT_NONE; S.lag_lo = S.est_lo; S.lag_hi = S.est_hi;
       est = 0;
     } else {
       const u32 c0 = 2u * y2, c1 = c0 + 1u;
@@ -614,7 +632,12 @@ __device__ __forceinline__ void dt_plan(DTop<K, V>& T, DtS& S, const u64 n_ops, 
   if (lag) {
     fl |= F_LAG;
     c->p_m[2][0] = S.lag_s0; c->p_m[2][1] = S.lag_s1;
-    c->p_m[2][2] = alloc(); c->p_m[2][3] = alloc();
+    if (S.lag_early) {  // G2 already split the staged children during the last phase B
+      fl |= F_LAGDONE;
+      c->p_m[2][2] = S.lag_lo; c->p_m[2][3] = S.lag_hi;
+    } else {
+      c->p_m[2][2] = alloc(); c->p_m[2][3] = alloc();
+    }
     c->p_sbi = S.lag_bi; c->p_spar = S.lag_par;
   }
   u32 rwait = 0, conflict = 0, m1v = 0, y1 = 0;
@@ -656,15 +679,8 @@ __device__ __forceinline__ void dt_plan(DTop<K, V>& T, DtS& S, const u64 n_ops, 
         y1 = 2u;
       }
       DT_MARK(3)
-      // take the refill node of op i+1 ahead (deep node, full-K op)
-      if (i + 1 < n_ops && C.n - (i + 1) * (u64)K >= (u64)K && hn >= DT_BIG) {
-        const u32 ps_ = alloc();
-        pre = 1; S.pre_tar = hn; S.pre_slot = ps_;
-        S.pre_bi = rbi; S.pre_par = (rph >> rbi) & 1u;
-        T.enqueue(RQ_REFILL, hn, ps_, rbi);
-        rph ^= 1u << rbi; rbi ^= 1u;
-      }
-      DT_MARK(4)
+      // (the STAGE for op i's depth-3 children goes first: G2 needs it this slot; the refill
+      // node of op i+1 is needed one slot later)
       if (y1) {
         const u32 cl = 2u * y1, cr = cl + 1u;
         const bool al = cl <= hn, ar = cr <= hn;
@@ -682,14 +698,30 @@ __device__ __forceinline__ void dt_plan(DTop<K, V>& T, DtS& S, const u64 n_ops, 
           const u32 p2 = (al && ar) ? (T.kmax(ncl) > T.kmax(ncr) ? cr : cl) : (al ? cl : cr);
           const u32 c0 = 2u * p2, c1 = c0 + 1u;
           if (c0 <= hn) {
+            const bool early = !(C.debug & 256u);  // test switch: split in the next phase A instead
             const u32 e0 = alloc(), e1 = alloc();
-            S.est = 1; S.est_y2 = p2; S.est_s0 = e0; S.est_s1 = e1;
+            const u32 elo = early ? alloc() : DT_NONE, ehi = early ? alloc() : DT_NONE;
+            S.est = 1; S.est_y2 = p2; S.est_s0 = e0; S.est_s1 = e1; S.est_lo = elo; S.est_hi = ehi;
             S.est_bi = sbi; S.est_par = (sph >> sbi) & 1u;
+            if (early) fl |= F_EARLY;
+            const u32 q = S.eseq + 1u;
+            S.eseq = q;
+            c->p_e[0] = e0; c->p_e[1] = e1; c->p_e[2] = elo; c->p_e[3] = ehi; c->p_e[4] = sbi; c->p_e[5] = S.est_par;
+            c->p_e[6] = q;
             T.enqueue(RQ_STAGE, c0, c1 <= H.cap ? c1 : 0u, e0, e1, sbi);
             sph ^= 1u << sbi; sbi ^= 1u;
           }
         }
       }
+      // take the refill node of op i+1 ahead (deep node, full-K op)
+      if (i + 1 < n_ops && C.n - (i + 1) * (u64)K >= (u64)K && hn >= DT_BIG) {
+        const u32 ps_ = alloc();
+        pre = 1; S.pre_tar = hn; S.pre_slot = ps_;
+        S.pre_bi = rbi; S.pre_par = (rph >> rbi) & 1u;
+        T.enqueue(RQ_REFILL, hn, ps_, rbi);
+        rph ^= 1u << rbi; rbi ^= 1u;
+      }
+      
       DT_MARK(5)
     }
   }
@@ -750,6 +782,8 @@ __device__ __forceinline__ void dt_top(DTop<K, V>& T) {
   for (;;) {
     const u32 pf = c->p_flags;
     if (pf == DT_NONE) break;
+    // plan words used after phase A: read now (thread 0 rewrites them during phase B)
+    const u32 w_sbi = c->p_sbi, w_spar = c->p_spar, w_rwait = c->p_rwait, w_rbi = c->p_rbi, w_rpar = c->p_rpar;
     if (tid == 0 && C.prog) C.prog[1] = 2;
     if (tid == 0 && ltime) { const ull t = clock64(); c->tm[0] += t - SS.tmark; SS.tmark = t; c->tm[5]++; if (SS.conflict) c->tm[6]++; }
 
@@ -795,7 +829,7 @@ __device__ __forceinline__ void dt_top(DTop<K, V>& T) {
                         T.BK(m[3]), T.BV(m[3]), mwin);
       }
     } else {
-      if (pf & F_LAG) {
+      if ((pf & F_LAG) && !(pf & F_LAGDONE)) {
         const u32 bi = c->p_sbi;
         const ull tw = (timing && gt == 0) ? clock64() : 0;
         mbar_wait(&c->sbar[bi], c->p_spar);
@@ -808,13 +842,27 @@ __device__ __forceinline__ void dt_top(DTop<K, V>& T) {
       }
     }
     if (timing && gt == 0) c->tm[8 + g] += clock64() - tg0;
+    // G2's early split of op i's staged depth-3 children (runs during phase B); its plan words
+    // are read before the barrier, after which thread 0 may plan the next slot
+    u32 e0 = 0, e1 = 0, elo = 0, ehi = 0, ebi = 0, epar = 0, eq = 0;
+    if (g == 2 && (pf & F_EARLY)) {
+      e0 = c->p_e[0]; e1 = c->p_e[1]; elo = c->p_e[2]; ehi = c->p_e[3]; ebi = c->p_e[4]; epar = c->p_e[5]; eq = c->p_e[6];
+    }
     cta_bar<DT_NTC>();
     if (tid == 0 && ltime) { const ull t = clock64(); c->tm[1] += t - SS.tmark; SS.tmark = t; }
     // every thread observes the TMA data phase B may read
     const ull tw7 = (tid == 0 && ltime) ? clock64() : 0;
-    if (pf & F_LAG) mbar_wait(&c->sbar[c->p_sbi], c->p_spar);
-    if (c->p_rwait) mbar_wait(&c->rbar[c->p_rbi], c->p_rpar);
+    if (pf & F_LAG) mbar_wait(&c->sbar[w_sbi], w_spar);
+    if (w_rwait) mbar_wait(&c->rbar[w_rbi], w_rpar);
     if (tid == 0 && ltime) c->ts[7] += clock64() - tw7;
+    if (g == 2 && (pf & F_EARLY)) {
+      mbar_wait(&c->sbar[ebi], epar);
+      if (c->stg_st[ebi][0] == ST_AVAIL && c->stg_st[ebi][1] == ST_AVAIL)
+        grp_split<K, V>(gt, T.BK(e0), T.BV(e0), K, T.BK(e1), T.BV(e1), K, K, T.BK(elo), T.BV(elo), T.BK(ehi),
+                        T.BV(ehi), mwin);
+      grp_bar(2);
+      if (gt == 0) st_rel_cta(&c->g2_done, eq);
+    }
     if (tid == 0 && timing) { const ull t = clock64(); c->tm[3] += t - SS.tmark; SS.tmark = t; }
 
     // =========================== phase B: decisions + job rounds ===========================
@@ -1062,11 +1110,13 @@ __device__ __forceinline__ void dt_top(DTop<K, V>& T) {
               break;
             }
             case 8: {
+              S.lag_early = 0;
               if (S.walk2) {
                 S.lag = true; S.lag_cur = S.y2;
                 const u32 c0 = 2u * S.y2, c1 = c0 + 1u;
                 if (S.est && S.est_y2 == S.y2) {
                   S.lag_bi = S.est_bi; S.lag_par = S.est_par; S.lag_s0 = S.est_s0; S.lag_s1 = S.est_s1;
+                  S.lag_early = S.est_lo != DT_NONE; S.lag_lo = S.est_lo; S.lag_hi = S.est_hi;
                   S.est = false;
                 } else {
                   S.lag_s0 = T.alloc(S); S.lag_s1 = T.alloc(S);
@@ -1082,7 +1132,10 @@ __device__ __forceinline__ void dt_top(DTop<K, V>& T) {
               if (S.est) {  // the walk stopped above depth 2: UNLOCK the staged children
                 T.enqueue(RQ_WB, 2u * S.est_y2, 2u * S.est_y2 + 1u <= H.cap ? 2u * S.est_y2 + 1u : 0u, 0u);
                 mbar_wait(&c->sbar[S.est_bi], S.est_par);  // the staging TMA must land before reuse
+                if (S.est_lo != DT_NONE)
+                  while (*reinterpret_cast<volatile u32*>(&c->g2_done) != S.eseq) __nanosleep(32);  // and G2's split
                 T.release_slot(S, S.est_s0); T.release_slot(S, S.est_s1);
+                T.release_slot(S, S.est_lo); T.release_slot(S, S.est_hi);
                 S.est = false;
               }
               if (S.fl & F_NEW) ++S.i;
@@ -1302,7 +1355,8 @@ __global__ void __launch_bounds__(DT_BLOCK, 1) bgpq_dtop_kernel(HeapArgs H, Call
       mbar_init(&c->sbar[0], 1); mbar_init(&c->sbar[1], 1);
       mbar_init(&c->rbar[0], 1); mbar_init(&c->rbar[1], 1);
       mbar_init(&c->lbar, 1);
-      c->rq_head[0] = c->rq_head[1] = 0; c->rq_done[0] = c->rq_done[1] = 0; c->tasks = 0; c->njobs = 0; c->wb_rd = 0;
+      c->rq_head[0] = c->rq_head[1] = 0; c->rq_done[0] = c->rq_done[1] = 0; c->tasks = 0; c->g2_done = 0;
+      for (int q = 0; q < 2 * (int)DT_RQ; ++q) mbar_init(&c->qbar[q / DT_RQ][q % DT_RQ], 1); c->njobs = 0; c->wb_rd = 0;
       c->freemask = (1u << DT_NSLOT) - 1u;
       asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
