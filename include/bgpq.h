@@ -47,15 +47,23 @@ enum {
   BGPQ_FLAG_VALUES = 1u, /* store a uint32 value with every key (w = 8 B per entry)        */
   BGPQ_FLAG_SERIAL = 2u, /* execute operations one at a time on a single CTA (test mode:
                             the node layout then equals the sequential Alg.1-3 model)     */
-  BGPQ_FLAG_LOCKS = 4u,  /* paper-literal per-node-lock execution (the default; kept as an
-                            explicit flag for callers that name it)                        */
+  BGPQ_FLAG_LOCKS = 4u,  /* per-node-lock execution of every call (the mixed-call engine,
+                            used for insert-only and deletemin-only calls too)              */
   BGPQ_FLAG_SERVER = 8u  /* root-server execution: one CTA holds the root, the pBuffer and
                             the top levels in shared memory and executes every root section
                             in call order; workers run the lock walks below     */
 };
-/* Default execution: every CTA of a persistent grid executes whole operations (Alg.1, Alg.2+3)
- * with per-node locks taken top-down hand over hand; a lock warp per CTA takes
- * the next level's locks and stages its nodes while the CTA merges. */
+/* Default execution (no flag):
+ *  - bgpq_insert: a level pipeline — one CTA per heap depth applies that depth's
+ *    INSERT_HEAPIFY steps (Alg.1 l.30-34) in call order, the root stage runs PARTIAL_INSERT
+ *    (l.15-29), sorter CTAs run Sort(items) (l.2); the heap after the call equals the
+ *    sequential Alg.1 model node for node;
+ *  - bgpq_deletemin: a top CTA keeps the root, the pBuffer and depths 1-2 in shared memory,
+ *    runs every root section (Alg.2) and the depth-0..2 steps of Alg.3 in call order, and
+ *    hands the walk below depth 3 (node still locked) to walker CTAs that take the paper's
+ *    per-node locks top-down hand over hand;
+ *  - bgpq_run_mixed: every CTA of a persistent grid executes whole operations (Alg.1,
+ *    Alg.2+3) with per-node locks, a lock warp per CTA taking the next level's locks ahead. */
 
 /* Create an empty heap able to hold `capacity` keys with node capacity K (§3.1:
  * every non-root node holds K sorted keys; k > 1).  K must be one of 64, 128, 256, 512,

@@ -128,8 +128,9 @@ class BGPQ:
     def __init__(self, capacity: int, K: int = 1024, values: bool = True, serial: bool = False,
                  locks: bool = False, server: bool = False):
         """serial: one CTA, one operation at a time (layout equals the sequential model);
-        default (or locks=True): per-node-lock execution on all CTAs with a lock-ahead warp;
-        server: root-server execution."""
+        default: insert calls as a level pipeline, deletemin calls on a top CTA with walker
+        CTAs, mixed calls with per-node locks; locks=True: per-node-lock execution for every
+        call; server: root-server execution."""
         if K not in VALID_K:
             raise ValueError(f"K must be one of {VALID_K}")
         flags = ((FLAG_VALUES if values else 0) | (FLAG_SERIAL if serial else 0)

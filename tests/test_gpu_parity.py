@@ -37,7 +37,7 @@ MODES = ["default", "locks", "server"]
 
 
 def _mode(mode):
-    """default: INSERT calls as the level pipeline + lock-ahead DELETEMIN; locks: paper-literal
+    """default: INSERT calls as the level pipeline + top-CTA DELETEMIN with walkers; locks: paper-literal
     per-node locks for every call; server: root-server execution."""
     return {"locks": mode == "locks", "server": mode == "server"}
 
