@@ -41,7 +41,8 @@ namespace bgpqd {
 constexpr int DT_GT = 256;              // threads per merge group
 constexpr int DT_NG = 3;                // merge groups
 constexpr int DT_NTC = DT_GT * DT_NG;   // compute threads of the top CTA (= worker NT)
-constexpr int DT_BLOCK = DT_NTC + 64;   // + helper warps A, B (top) / lock warp + idle warp (workers)
+constexpr int DT_BLOCK = DT_NTC + 96;   // + control warp, helper warps A, B (top) / lock warp (walkers)
+constexpr int DT_BAR_READY = 6, DT_BAR_DONE = 7;  // named barriers: control warp <-> the 3 groups
 constexpr int DT_NSLOT = 28;            // smem node slots of the top CTA
 constexpr int DT_RQ = 16;               // helper request ring
 constexpr u32 DT_BIG = 64;              // pipelined mode needs heapSize >= DT_BIG
@@ -64,6 +65,8 @@ struct DtJob {
 // thread-0 state of the top CTA (see dt_top)
 struct DtS {
   u32 fm;  // free slot mask
+  u32 defer, ndq;        // control-warp driver: helper requests queued until the groups run
+  u32 dq[6][10];
   u32 eseq;              // early-split sequence number
   u32 est_lo, est_hi;    // output slots of the early depth-2 split of the staged children (G2, phase B)
   u32 lag_early, lag_lo, lag_hi;  // the pending lag step's split was done early into lag_lo / lag_hi
@@ -90,12 +93,6 @@ struct DtS {
   u32 est_par;
   u32 est_s0;
   u32 est_s1;
-  u32 wb0;
-  u32 wb1;
-  u32 wb_pub;
-  u32 wb_pending;
-  u32 fr0;
-  u32 fr1;
   u32 fl;
   u32 size;
   u32 path;
@@ -125,16 +122,16 @@ struct DtS {
   u32 walk2;
   u32 m1v;
   u32 conflict;
-  u32 lst;
   u64 i;
   u64 nout;
   u64 tmark;
   __device__ __forceinline__ void init() {
-    hs = 0; rs = 0; ps = 0; sph = 0; rph = 0; sbi = 0; rbi = 0; lag_cur = 0; lag_bi = 0; lag_par = 0; lag_s0 = 0; lag_s1 = 0; pre_tar = 0; pre_slot = 0; pre_bi = 0; pre_par = 0; est_y2 = 0; est_bi = 0; est_par = 0; est_s0 = 0; est_s1 = 0; wb0 = 0; wb1 = 0; wb_pub = 0; wb_pending = 0; fr0 = 0; fr1 = 0; fl = 0; size = 0; path = 0; R = 0; remained = 0; rs_old = 0; y1 = 0; y2 = 0; car1 = 0; m1lo = 0; m1hi = 0; mfa = 0; mfb = 0; tsl = 0; lx = 0; ly = 0; lX = 0; lcar = 0; lcar3 = 0; lcf = 0; take_sv = 0; stage = 0; lag = 0; pre = 0; est = 0; walk = 0; walk2 = 0; m1v = 0; conflict = 0; lst = 0; i = 0; nout = 0; tmark = 0;
+    hs = 0; rs = 0; ps = 0; sph = 0; rph = 0; sbi = 0; rbi = 0; lag_cur = 0; lag_bi = 0; lag_par = 0; lag_s0 = 0; lag_s1 = 0; pre_tar = 0; pre_slot = 0; pre_bi = 0; pre_par = 0; est_y2 = 0; est_bi = 0; est_par = 0; est_s0 = 0; est_s1 = 0; fl = 0; size = 0; path = 0; R = 0; remained = 0; rs_old = 0; y1 = 0; y2 = 0; car1 = 0; m1lo = 0; m1hi = 0; mfa = 0; mfb = 0; tsl = 0; lx = 0; ly = 0; lX = 0; lcar = 0; lcar3 = 0; lcf = 0; take_sv = 0; stage = 0; lag = 0; pre = 0; est = 0; walk = 0; walk2 = 0; m1v = 0; conflict = 0; i = 0; nout = 0; tmark = 0;
     pout = pout_old = DT_NONE;
+    defer = 0; ndq = 0;
     est_lo = est_hi = lag_lo = lag_hi = DT_NONE; lag_early = 0;
     wbs = pq0 = pq1 = 0; pa0 = pb0 = pa1 = pb1 = DT_NONE;
-    fr0 = fr1 = car1 = m1lo = m1hi = mfa = mfb = tsl = lX = lcar = lcar3 = lcf = R = DT_NONE;
+    car1 = m1lo = m1hi = mfa = mfb = tsl = lX = lcar = lcar3 = lcf = R = DT_NONE;
   }
 };
 
@@ -156,6 +153,7 @@ struct DtCtl {
   u32 p_out_slot, p_out_n, p_iop_lo, p_iop_hi;
   u32 p_m[3][4]; // group g: split slots z, w -> lo, hi
   u32 p_sbi, p_spar, p_rwait, p_rbi, p_rpar;
+  u32 ctl_done;  // control warp: the slot's decisions are complete
   u32 g2_done;   // G2: sequence number of the last early split finished
   u32 p_e[7];    // early depth-2 split for G2 in phase B: staged s0, s1 -> lo, hi; sbar index, parity
   u32 more;      // another job round follows
@@ -166,9 +164,10 @@ struct DtCtl {
   ull ts[12];    // debug: thread-0 cycles per phase-B stage
   ull tm[12];    // debug timers (C.debug & 8): plan, phase A, G2 stage wait, refill wait, phase B, slots, conflicts, helper lock wait
 };
-enum : u32 { F_NEW = 1, F_LAG = 2, F_M0 = 4, F_M1 = 8, F_LAGDONE = 16, F_EARLY = 32 };
+enum : u32 { F_NEW = 1, F_LAG = 2, F_M0 = 4, F_M1 = 8, F_LAGDONE = 16, F_EARLY = 32, F_JOBS = 64 };
 constexpr size_t DTCTL_BYTES = (sizeof(DtCtl) + 127) / 128 * 128;
 
+static_assert(DTCTL_BYTES + (size_t)DT_NSLOT * 1024 * 4 * 2 <= 232448, "top CTA exceeds 227 KB of shared memory at K=1024 w=8");
 template <int K, bool V>
 constexpr size_t dt_smem_bytes() {
   const size_t top = DTCTL_BYTES + (size_t)DT_NSLOT * K * 4 * (V ? 2 : 1);
@@ -245,6 +244,22 @@ struct DTop {
     asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_addr(&c->qbar[r][h % DT_RQ])) : "memory");
     if (C.debug & 8u) c->ts[9] += clock64() - tq;
   }
+  // ---- a helper request now, or (control-warp driver) after the groups were released
+  __device__ __forceinline__ void req(DtS& S, u32 type, u32 a0 = 0, u32 a1 = 0, u32 a2 = 0, u32 a3 = 0, u32 a4 = 0,
+                                      u32 a5 = 0, u32 a6 = 0, u32 a7 = 0, u32 a8 = 0) {
+    if (!S.defer) { enqueue(type, a0, a1, a2, a3, a4, a5, a6, a7, a8); return; }
+    u32* e = S.dq[S.ndq++];
+    e[0] = type; e[1] = a0; e[2] = a1; e[3] = a2; e[4] = a3; e[5] = a4; e[6] = a5; e[7] = a6; e[8] = a7; e[9] = a8;
+  }
+  __device__ __forceinline__ void flush(DtS& S) {
+    const u32 n = S.ndq;
+    for (u32 q = 0; q < n; ++q) {
+      const u32* e = S.dq[q];
+      enqueue(e[0], e[1], e[2], e[3], e[4], e[5], e[6], e[7], e[8], e[9]);
+    }
+    S.ndq = 0;
+  }
+
   // ---- thread 0: hand the write-back of a lag step to the helper (RQ_WB2): node x <- slot X
   // (X = DT_NONE: only UNLOCK x), node y <- slot Y, then UNLOCK x and publish y to a walker
   // (pub) or UNLOCK it.  The slots stay allocated until the helper has read them (wb_rd).
@@ -502,8 +517,8 @@ __device__ __forceinline__ bool dt_fast(DTop<K, V>& T, DtS& S) {
     fm |= (1u << lag_s0) | (1u << lag_s1);
     const u32 seq = S.wbs + 1u;
     S.wbs = seq;
-    T.enqueue(RQ_WB2, x3, hi2, y3, lcar, ((2u * y3 <= hs0) ? 1u : 0u) | (seq << 1), T.kmin(hi2), T.kmax(hi2),
-              lcarmin, lcarmax);
+    T.req(S, RQ_WB2, x3, hi2, y3, lcar, ((2u * y3 <= hs0) ? 1u : 0u) | (seq << 1), T.kmin(hi2), T.kmax(hi2),
+          lcarmin, lcarmax);
     // slots of the write-back two generations ago: free once helper B has read them
     const u32 pq1 = S.pq1;
     if (pq1 != 0) {
@@ -568,7 +583,7 @@ __device__ __forceinline__ bool dt_fast(DTop<K, V>& T, DtS& S) {
       const u32 sbi = S.sbi, sph = S.sph;
       S.lag_s0 = sa; S.lag_s1 = sb;
       S.lag_bi = sbi; S.lag_par = (sph >> sbi) & 1u;
-      T.enqueue(RQ_STAGE, c0, c1 <= H.cap ? c1 : 0u, sa, sb, sbi);
+      T.req(S, RQ_STAGE, c0, c1 <= H.cap ? c1 : 0u, sa, sb, sbi);
       S.sph = sph ^ (1u << sbi); S.sbi = sbi ^ 1u;
     }
   }
@@ -662,7 +677,7 @@ __device__ __forceinline__ void dt_plan(DTop<K, V>& T, DtS& S, const u64 n_ops, 
         c->ns[hs] = DT_NONE;
       } else {  // synchronous take by the helper
         R = alloc();
-        T.enqueue(RQ_REFILL, hs, R, rbi);
+        T.req(S, RQ_REFILL, hs, R, rbi);
         rwait = 1; c->p_rbi = rbi; c->p_rpar = (rph >> rbi) & 1u;
         rph ^= 1u << rbi; rbi ^= 1u;
       }
@@ -698,7 +713,7 @@ __device__ __forceinline__ void dt_plan(DTop<K, V>& T, DtS& S, const u64 n_ops, 
           const u32 p2 = (al && ar) ? (T.kmax(ncl) > T.kmax(ncr) ? cr : cl) : (al ? cl : cr);
           const u32 c0 = 2u * p2, c1 = c0 + 1u;
           if (c0 <= hn) {
-            const bool early = !(C.debug & 256u);  // test switch: split in the next phase A instead
+            const bool early = !(C.debug & 256u) && !S.defer;  // (control-warp driver: split in phase A)
             const u32 e0 = alloc(), e1 = alloc();
             const u32 elo = early ? alloc() : DT_NONE, ehi = early ? alloc() : DT_NONE;
             S.est = 1; S.est_y2 = p2; S.est_s0 = e0; S.est_s1 = e1; S.est_lo = elo; S.est_hi = ehi;
@@ -708,7 +723,7 @@ __device__ __forceinline__ void dt_plan(DTop<K, V>& T, DtS& S, const u64 n_ops, 
             S.eseq = q;
             c->p_e[0] = e0; c->p_e[1] = e1; c->p_e[2] = elo; c->p_e[3] = ehi; c->p_e[4] = sbi; c->p_e[5] = S.est_par;
             c->p_e[6] = q;
-            T.enqueue(RQ_STAGE, c0, c1 <= H.cap ? c1 : 0u, e0, e1, sbi);
+            T.req(S, RQ_STAGE, c0, c1 <= H.cap ? c1 : 0u, e0, e1, sbi);
             sph ^= 1u << sbi; sbi ^= 1u;
           }
         }
@@ -718,7 +733,7 @@ __device__ __forceinline__ void dt_plan(DTop<K, V>& T, DtS& S, const u64 n_ops, 
         const u32 ps_ = alloc();
         pre = 1; S.pre_tar = hn; S.pre_slot = ps_;
         S.pre_bi = rbi; S.pre_par = (rph >> rbi) & 1u;
-        T.enqueue(RQ_REFILL, hn, ps_, rbi);
+        T.req(S, RQ_REFILL, hn, ps_, rbi);
         rph ^= 1u << rbi; rbi ^= 1u;
       }
       
@@ -733,147 +748,13 @@ __device__ __forceinline__ void dt_plan(DTop<K, V>& T, DtS& S, const u64 n_ops, 
   DT_MARK(6)
 }
 
+// Phase B general path (thread 0): Alg.2/Alg.3 as a state machine; returns when it posted a
+// collective job list (merges, copies) for the compute threads or finished the slot.
 template <int K, bool V>
-__device__ __forceinline__ void dt_top(DTop<K, V>& T) {
+__device__ __forceinline__ bool dt_slow(DTop<K, V>& T, DtS& S, const bool timing) {
   DtCtl* c = T.c;
   const HeapArgs& H = T.H;
-  const CallArgs& C = T.C;
-  const int tid = threadIdx.x;
-  const int g = tid / DT_GT, gt = tid % DT_GT;
-  const u64 n_ops = C.n_ops;
-  constexpr u32 NBY = K * 4u;
-  // ---- thread-0 state lives in shared memory (DtS): the helper warp's gpu-scope acquires
-  // invalidate L1, so registers spilled to local memory would cost an L2 round trip each
-  DtS& SS = c->s;
-  if (tid == 0) { SS.init(); SS.fm = (1u << DT_NSLOT) - 1u; }
-  // ---- call start: stage the on-chip part (pBuffer, root, nodes 2..7)
-  if (tid == 0) {
-    DtS* __restrict__ const Sp = &SS;
-    DtS& S = *Sp;
-    S.hs = ld_relaxed(H.hdr + H_HS);
-    S.rs = ld_relaxed(H.hdr + H_RS);
-    S.ps = ld_relaxed(H.hdr + H_PS);
-    u32 bytes = 0;
-    for (u32 q = 0; q < 8; ++q) {
-      const bool have = q == 0 ? S.ps > 0 : (q == 1 ? (S.hs >= 1 && S.rs > 0) : q <= S.hs);
-      c->ns[q] = have ? T.alloc(S) : DT_NONE;
-      if (have) bytes += V ? 2u * NBY : NBY;
-    }
-    fence_proxy_async();
-    mbar_arrive_expect_tx(&c->lbar, bytes);
-    for (u32 q = 0; q < 8; ++q) {
-      if (c->ns[q] == DT_NONE) continue;
-      bulk_g2s(T.BK(c->ns[q]), H.gk + (size_t)q * K, NBY, &c->lbar);
-      if (V) bulk_g2s(T.BV(c->ns[q]), H.gv + (size_t)q * K, NBY, &c->lbar);
-    }
-    (void)0;
-  }
-  mbar_wait(&c->lbar, 0);
-  cta_bar<DT_NTC>();
-
-  const bool timing = (C.debug & 8u) != 0;
-  const bool ltime = timing || (C.debug & 128u) != 0;  // light timing: plan / phase A / phase B only
-  const bool mwin = (C.debug & 64u) != 0;
-  // the first plan; every later one is made by thread 0 at the end of the previous slot's
-  // phase B, so a common slot has two CTA barriers (after phase A, after phase B)
-  if (tid == 0 && ltime) SS.tmark = clock64();
-  if (tid == 0) dt_plan<K, V>(T, SS, n_ops, timing);
-  cta_bar<DT_NTC>();
-  for (;;) {
-    const u32 pf = c->p_flags;
-    if (pf == DT_NONE) break;
-    // plan words used after phase A: read now (thread 0 rewrites them during phase B)
-    const u32 w_sbi = c->p_sbi, w_spar = c->p_spar, w_rwait = c->p_rwait, w_rbi = c->p_rbi, w_rpar = c->p_rpar;
-    if (tid == 0 && C.prog) C.prog[1] = 2;
-    if (tid == 0 && ltime) { const ull t = clock64(); c->tm[0] += t - SS.tmark; SS.tmark = t; c->tm[5]++; if (SS.conflict) c->tm[6]++; }
-
-    // =========================== phase A: concurrent work ===========================
-    const ull tg0 = (timing && gt == 0) ? clock64() : 0;
-    if (g == 0) {
-      if (pf & F_NEW) {  // Alg.2 l.18-22: the old root keys are the first output of op i
-        const u32 n = c->p_out_n;
-        const u64 pos0 = (((u64)c->p_iop_hi << 32) | c->p_iop_lo) * (u64)K;
-        const bool bulk = (n & 3u) == 0 && ((reinterpret_cast<uintptr_t>(C.out_k + pos0) & 15u) == 0) &&
-                          (!V || !C.out_v || (reinterpret_cast<uintptr_t>(C.out_v + pos0) & 15u) == 0);
-        if (n && bulk) {  // one TMA bulk store (async proxy); its smem read is awaited before the slot is reused
-          if (gt == 0) {
-            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-            bulk_s2g(C.out_k + pos0, T.BK(c->p_out_slot), n * 4u);
-            if (V && C.out_v) bulk_s2g(C.out_v + pos0, T.BV(c->p_out_slot), n * 4u);
-            asm volatile("cp.async.bulk.commit_group;" ::: "memory");
-          }
-        } else if (n) {
-          const u64 pos = (((u64)c->p_iop_hi << 32) | c->p_iop_lo) * (u64)K;
-          const u32* s = T.BK(c->p_out_slot);
-          if ((n & 3u) == 0) {
-            uint4* d4 = reinterpret_cast<uint4*>(C.out_k + pos);
-            for (u32 q = gt; q < n / 4; q += DT_GT) d4[q] = reinterpret_cast<const uint4*>(s)[q];
-          } else {
-            for (u32 q = gt; q < n; q += DT_GT) C.out_k[pos + q] = s[q];
-          }
-          if (V && C.out_v) {
-            const u32* v = T.BV(c->p_out_slot);
-            for (u32 q = gt; q < n; q += DT_GT) C.out_v[pos + q] = v[q];
-          }
-        }
-      }
-      if (pf & F_M0) {
-        const u32* m = c->p_m[0];
-        grp_split<K, V>(gt, T.BK(m[0]), T.BV(m[0]), K, T.BK(m[1]), T.BV(m[1]), K, K, T.BK(m[2]), T.BV(m[2]),
-                        T.BK(m[3]), T.BV(m[3]), mwin);
-      }
-    } else if (g == 1) {
-      if (pf & F_M1) {
-        const u32* m = c->p_m[1];
-        grp_split<K, V>(gt, T.BK(m[0]), T.BV(m[0]), K, T.BK(m[1]), T.BV(m[1]), K, K, T.BK(m[2]), T.BV(m[2]),
-                        T.BK(m[3]), T.BV(m[3]), mwin);
-      }
-    } else {
-      if ((pf & F_LAG) && !(pf & F_LAGDONE)) {
-        const u32 bi = c->p_sbi;
-        const ull tw = (timing && gt == 0) ? clock64() : 0;
-        mbar_wait(&c->sbar[bi], c->p_spar);
-        if (timing && gt == 0) c->tm[2] += clock64() - tw;
-        if (c->stg_st[bi][0] == ST_AVAIL && c->stg_st[bi][1] == ST_AVAIL) {
-          const u32* m = c->p_m[2];
-          grp_split<K, V>(gt, T.BK(m[0]), T.BV(m[0]), K, T.BK(m[1]), T.BV(m[1]), K, K, T.BK(m[2]), T.BV(m[2]),
-                          T.BK(m[3]), T.BV(m[3]), mwin);
-        }
-      }
-    }
-    if (timing && gt == 0) c->tm[8 + g] += clock64() - tg0;
-    // G2's early split of op i's staged depth-3 children (runs during phase B); its plan words
-    // are read before the barrier, after which thread 0 may plan the next slot
-    u32 e0 = 0, e1 = 0, elo = 0, ehi = 0, ebi = 0, epar = 0, eq = 0;
-    if (g == 2 && (pf & F_EARLY)) {
-      e0 = c->p_e[0]; e1 = c->p_e[1]; elo = c->p_e[2]; ehi = c->p_e[3]; ebi = c->p_e[4]; epar = c->p_e[5]; eq = c->p_e[6];
-    }
-    cta_bar<DT_NTC>();
-    if (tid == 0 && ltime) { const ull t = clock64(); c->tm[1] += t - SS.tmark; SS.tmark = t; }
-    // every thread observes the TMA data phase B may read
-    const ull tw7 = (tid == 0 && ltime) ? clock64() : 0;
-    if (pf & F_LAG) mbar_wait(&c->sbar[w_sbi], w_spar);
-    if (w_rwait) mbar_wait(&c->rbar[w_rbi], w_rpar);
-    if (tid == 0 && ltime) c->ts[7] += clock64() - tw7;
-    if (g == 2 && (pf & F_EARLY)) {
-      mbar_wait(&c->sbar[ebi], epar);
-      if (c->stg_st[ebi][0] == ST_AVAIL && c->stg_st[ebi][1] == ST_AVAIL)
-        grp_split<K, V>(gt, T.BK(e0), T.BV(e0), K, T.BK(e1), T.BV(e1), K, K, T.BK(elo), T.BV(elo), T.BK(ehi),
-                        T.BV(ehi), mwin);
-      grp_bar(2);
-      if (gt == 0) st_rel_cta(&c->g2_done, eq);
-    }
-    if (tid == 0 && timing) { const ull t = clock64(); c->tm[3] += t - SS.tmark; SS.tmark = t; }
-
-    // =========================== phase B: decisions + job rounds ===========================
-    if (tid == 0) SS.stage = 0;
-    for (;;) {
-      if (tid == 0) {
-        DtS* __restrict__ const Sp = &SS;
-        DtS& S = *Sp;
-        c->njobs = 0;
-        bool done = false;
-        if (S.stage == 0) done = dt_fast<K, V>(T, S);  // the common slot, straight-line
+  bool done = false;
         while (c->njobs == 0 && !done) {
           const u32 st_in = S.stage;
           const ull tsw = timing ? clock64() : 0;
@@ -1145,6 +1026,151 @@ __device__ __forceinline__ void dt_top(DTop<K, V>& T) {
           }
           if (timing) c->ts[st_in >= 30 ? 8 : (st_in > 8 ? 8 : st_in)] += clock64() - tsw;
         }
+  return done;
+}
+
+template <int K, bool V>
+__device__ __forceinline__ void dt_top(DTop<K, V>& T) {
+  DtCtl* c = T.c;
+  const HeapArgs& H = T.H;
+  const CallArgs& C = T.C;
+  const int tid = threadIdx.x;
+  const int g = tid / DT_GT, gt = tid % DT_GT;
+  const u64 n_ops = C.n_ops;
+  constexpr u32 NBY = K * 4u;
+  // ---- thread-0 state lives in shared memory (DtS): the helper warp's gpu-scope acquires
+  // invalidate L1, so registers spilled to local memory would cost an L2 round trip each
+  DtS& SS = c->s;
+  if (tid == 0) { SS.init(); SS.fm = (1u << DT_NSLOT) - 1u; }
+  // ---- call start: stage the on-chip part (pBuffer, root, nodes 2..7)
+  if (tid == 0) {
+    DtS* __restrict__ const Sp = &SS;
+    DtS& S = *Sp;
+    S.hs = ld_relaxed(H.hdr + H_HS);
+    S.rs = ld_relaxed(H.hdr + H_RS);
+    S.ps = ld_relaxed(H.hdr + H_PS);
+    u32 bytes = 0;
+    for (u32 q = 0; q < 8; ++q) {
+      const bool have = q == 0 ? S.ps > 0 : (q == 1 ? (S.hs >= 1 && S.rs > 0) : q <= S.hs);
+      c->ns[q] = have ? T.alloc(S) : DT_NONE;
+      if (have) bytes += V ? 2u * NBY : NBY;
+    }
+    fence_proxy_async();
+    mbar_arrive_expect_tx(&c->lbar, bytes);
+    for (u32 q = 0; q < 8; ++q) {
+      if (c->ns[q] == DT_NONE) continue;
+      bulk_g2s(T.BK(c->ns[q]), H.gk + (size_t)q * K, NBY, &c->lbar);
+      if (V) bulk_g2s(T.BV(c->ns[q]), H.gv + (size_t)q * K, NBY, &c->lbar);
+    }
+    (void)0;
+  }
+  mbar_wait(&c->lbar, 0);
+  cta_bar<DT_NTC>();
+
+  const bool timing = (C.debug & 8u) != 0;
+  const bool ltime = timing || (C.debug & 128u) != 0;  // light timing: plan / phase A / phase B only
+  const bool mwin = (C.debug & 64u) != 0;
+  // the first plan; every later one is made by thread 0 at the end of the previous slot's
+  // phase B, so a common slot has two CTA barriers (after phase A, after phase B)
+  if (tid == 0 && ltime) SS.tmark = clock64();
+  if (tid == 0) dt_plan<K, V>(T, SS, n_ops, timing);
+  cta_bar<DT_NTC>();
+  for (;;) {
+    const u32 pf = c->p_flags;
+    if (pf == DT_NONE) break;
+    // plan words used after phase A: read now (thread 0 rewrites them during phase B)
+    const u32 w_sbi = c->p_sbi, w_spar = c->p_spar, w_rwait = c->p_rwait, w_rbi = c->p_rbi, w_rpar = c->p_rpar;
+    if (tid == 0 && C.prog) C.prog[1] = 2;
+    if (tid == 0 && ltime) { const ull t = clock64(); c->tm[0] += t - SS.tmark; SS.tmark = t; c->tm[5]++; if (SS.conflict) c->tm[6]++; }
+
+    // =========================== phase A: concurrent work ===========================
+    const ull tg0 = (timing && gt == 0) ? clock64() : 0;
+    if (g == 0) {
+      if (pf & F_NEW) {  // Alg.2 l.18-22: the old root keys are the first output of op i
+        const u32 n = c->p_out_n;
+        const u64 pos0 = (((u64)c->p_iop_hi << 32) | c->p_iop_lo) * (u64)K;
+        const bool bulk = (n & 3u) == 0 && ((reinterpret_cast<uintptr_t>(C.out_k + pos0) & 15u) == 0) &&
+                          (!V || !C.out_v || (reinterpret_cast<uintptr_t>(C.out_v + pos0) & 15u) == 0);
+        if (n && bulk) {  // one TMA bulk store (async proxy); its smem read is awaited before the slot is reused
+          if (gt == 0) {
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            bulk_s2g(C.out_k + pos0, T.BK(c->p_out_slot), n * 4u);
+            if (V && C.out_v) bulk_s2g(C.out_v + pos0, T.BV(c->p_out_slot), n * 4u);
+            asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+          }
+        } else if (n) {
+          const u64 pos = (((u64)c->p_iop_hi << 32) | c->p_iop_lo) * (u64)K;
+          const u32* s = T.BK(c->p_out_slot);
+          if ((n & 3u) == 0) {
+            uint4* d4 = reinterpret_cast<uint4*>(C.out_k + pos);
+            for (u32 q = gt; q < n / 4; q += DT_GT) d4[q] = reinterpret_cast<const uint4*>(s)[q];
+          } else {
+            for (u32 q = gt; q < n; q += DT_GT) C.out_k[pos + q] = s[q];
+          }
+          if (V && C.out_v) {
+            const u32* v = T.BV(c->p_out_slot);
+            for (u32 q = gt; q < n; q += DT_GT) C.out_v[pos + q] = v[q];
+          }
+        }
+      }
+      if (pf & F_M0) {
+        const u32* m = c->p_m[0];
+        grp_split<K, V>(gt, T.BK(m[0]), T.BV(m[0]), K, T.BK(m[1]), T.BV(m[1]), K, K, T.BK(m[2]), T.BV(m[2]),
+                        T.BK(m[3]), T.BV(m[3]), mwin);
+      }
+    } else if (g == 1) {
+      if (pf & F_M1) {
+        const u32* m = c->p_m[1];
+        grp_split<K, V>(gt, T.BK(m[0]), T.BV(m[0]), K, T.BK(m[1]), T.BV(m[1]), K, K, T.BK(m[2]), T.BV(m[2]),
+                        T.BK(m[3]), T.BV(m[3]), mwin);
+      }
+    } else {
+      if ((pf & F_LAG) && !(pf & F_LAGDONE)) {
+        const u32 bi = c->p_sbi;
+        const ull tw = (timing && gt == 0) ? clock64() : 0;
+        mbar_wait(&c->sbar[bi], c->p_spar);
+        if (timing && gt == 0) c->tm[2] += clock64() - tw;
+        if (c->stg_st[bi][0] == ST_AVAIL && c->stg_st[bi][1] == ST_AVAIL) {
+          const u32* m = c->p_m[2];
+          grp_split<K, V>(gt, T.BK(m[0]), T.BV(m[0]), K, T.BK(m[1]), T.BV(m[1]), K, K, T.BK(m[2]), T.BV(m[2]),
+                          T.BK(m[3]), T.BV(m[3]), mwin);
+        }
+      }
+    }
+    if (timing && gt == 0) c->tm[8 + g] += clock64() - tg0;
+    // G2's early split of op i's staged depth-3 children (runs during phase B); its plan words
+    // are read before the barrier, after which thread 0 may plan the next slot
+    u32 e0 = 0, e1 = 0, elo = 0, ehi = 0, ebi = 0, epar = 0, eq = 0;
+    if (g == 2 && (pf & F_EARLY)) {
+      e0 = c->p_e[0]; e1 = c->p_e[1]; elo = c->p_e[2]; ehi = c->p_e[3]; ebi = c->p_e[4]; epar = c->p_e[5]; eq = c->p_e[6];
+    }
+    cta_bar<DT_NTC>();
+    if (tid == 0 && ltime) { const ull t = clock64(); c->tm[1] += t - SS.tmark; SS.tmark = t; }
+    // every thread observes the TMA data phase B may read
+    const ull tw7 = (tid == 0 && ltime) ? clock64() : 0;
+    if (pf & F_LAG) mbar_wait(&c->sbar[w_sbi], w_spar);
+    if (w_rwait) mbar_wait(&c->rbar[w_rbi], w_rpar);
+    if (tid == 0 && ltime) c->ts[7] += clock64() - tw7;
+    if (g == 2 && (pf & F_EARLY)) {
+      mbar_wait(&c->sbar[ebi], epar);
+      if (c->stg_st[ebi][0] == ST_AVAIL && c->stg_st[ebi][1] == ST_AVAIL)
+        grp_split<K, V>(gt, T.BK(e0), T.BV(e0), K, T.BK(e1), T.BV(e1), K, K, T.BK(elo), T.BV(elo), T.BK(ehi),
+                        T.BV(ehi), mwin);
+      grp_bar(2);
+      if (gt == 0) st_rel_cta(&c->g2_done, eq);
+    }
+    if (tid == 0 && timing) { const ull t = clock64(); c->tm[3] += t - SS.tmark; SS.tmark = t; }
+
+    // =========================== phase B: decisions + job rounds ===========================
+    if (tid == 0) SS.stage = 0;
+    for (;;) {
+      if (tid == 0) {
+        DtS* __restrict__ const Sp = &SS;
+        DtS& S = *Sp;
+        c->njobs = 0;
+        bool done = false;
+        if (S.stage == 0) done = dt_fast<K, V>(T, S);  // the common slot, straight-line
+        if (!done) done = dt_slow<K, V>(T, S, timing);
         if (done) {  // the slot is complete: plan the next one now
           if (ltime) { const ull t = clock64(); c->tm[4] += t - SS.tmark; SS.tmark = t; }
           dt_plan<K, V>(T, SS, n_ops, timing);
@@ -1208,6 +1234,212 @@ __device__ __forceinline__ void dt_top(DTop<K, V>& T) {
     }
     (void)0;
   }
+}
+
+// named barriers (aligned forms: the whole warp must execute them convergently, hence the
+// __syncwarp after any lane-0-only code)
+__device__ __forceinline__ void nbar_sync(int id, int n) {
+  __syncwarp();
+  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory");
+}
+__device__ __forceinline__ void nbar_arrive(int id, int n) {
+  __syncwarp();
+  asm volatile("bar.arrive %0, %1;" ::"r"(id), "r"(n) : "memory");
+}
+
+// =========================================================================================
+// Control-warp driver (test switch BGPQ_DEBUG bit 512; measured no faster than dt_top, whose
+// thread-0 decision chain it moves to a dedicated warp).  The decisions of a slot (dt_fast / dt_slow, then dt_plan)
+// run on a dedicated warp: the three groups are released (barrier READY) as soon as the plan
+// of the next slot is written, and the control warp then issues the slot's helper requests and
+// the output copy while the groups merge; the groups report phase A done on barrier DONE.
+// =========================================================================================
+template <int K, bool V>
+__device__ __forceinline__ void dt_groups2(DTop<K, V>& T) {
+  DtCtl* c = T.c;
+  const int tid = threadIdx.x, g = tid / DT_GT, gt = tid % DT_GT;
+  const bool mwin = (T.C.debug & 64u) != 0;
+  constexpr int NB_ = DT_NTC + 32;
+  mbar_wait(&c->lbar, 0);
+  for (;;) {
+    nbar_sync(DT_BAR_READY, NB_);
+    const u32 pf = c->p_flags;
+    if (pf == DT_NONE) break;
+    if (pf & F_JOBS) {
+      T.run_jobs();
+      nbar_arrive(DT_BAR_DONE, NB_);
+      continue;
+    }
+    const u32 w_sbi = c->p_sbi, w_spar = c->p_spar, w_rwait = c->p_rwait, w_rbi = c->p_rbi, w_rpar = c->p_rpar;
+    const bool lt = (T.C.debug & 128u) != 0;
+    const ull ta = (lt && gt == 0) ? clock64() : 0;
+    if (g == 0 && (pf & F_M0)) {
+      const u32* m = c->p_m[0];
+      grp_split<K, V>(gt, T.BK(m[0]), T.BV(m[0]), K, T.BK(m[1]), T.BV(m[1]), K, K, T.BK(m[2]), T.BV(m[2]),
+                      T.BK(m[3]), T.BV(m[3]), mwin);
+    }
+    if (g == 1 && (pf & F_M1)) {
+      const u32* m = c->p_m[1];
+      grp_split<K, V>(gt, T.BK(m[0]), T.BV(m[0]), K, T.BK(m[1]), T.BV(m[1]), K, K, T.BK(m[2]), T.BV(m[2]),
+                      T.BK(m[3]), T.BV(m[3]), mwin);
+    }
+    if (g == 2 && (pf & F_LAG) && !(pf & F_LAGDONE)) {
+      mbar_wait(&c->sbar[w_sbi], w_spar);
+      if (c->stg_st[w_sbi][0] == ST_AVAIL && c->stg_st[w_sbi][1] == ST_AVAIL) {
+        const u32* m = c->p_m[2];
+        grp_split<K, V>(gt, T.BK(m[0]), T.BV(m[0]), K, T.BK(m[1]), T.BV(m[1]), K, K, T.BK(m[2]), T.BV(m[2]),
+                        T.BK(m[3]), T.BV(m[3]), mwin);
+      }
+    }
+    if (lt && gt == 0) c->tm[8 + g] += clock64() - ta;
+    // the TMA data the control warp reads next (staged children, refill node) has landed
+    const ull tw = (lt && gt == 0) ? clock64() : 0;
+    if (pf & F_LAG) mbar_wait(&c->sbar[w_sbi], w_spar);
+    if (w_rwait) mbar_wait(&c->rbar[w_rbi], w_rpar);
+    if (lt && gt == 0) c->tm[3] += clock64() - tw;
+    nbar_arrive(DT_BAR_DONE, NB_);
+  }
+}
+
+// control warp, lane 0 works; the whole warp takes part in the named barriers
+template <int K, bool V>
+__device__ __forceinline__ void dt_control(DTop<K, V>& T) {
+  DtCtl* c = T.c;
+  const HeapArgs& H = T.H;
+  const CallArgs& C = T.C;
+  const u32 lane = threadIdx.x & 31;
+  const u64 n_ops = C.n_ops;
+  constexpr u32 NBY = K * 4u;
+  constexpr int NB_ = DT_NTC + 32;
+  DtS& SS = c->s;
+  if (lane == 0) {
+    DtS* __restrict__ const Sp = &SS;
+    DtS& S = *Sp;
+    S.init();
+    S.fm = (1u << DT_NSLOT) - 1u;
+    S.defer = 1;
+    S.hs = ld_relaxed(H.hdr + H_HS);
+    S.rs = ld_relaxed(H.hdr + H_RS);
+    S.ps = ld_relaxed(H.hdr + H_PS);
+    u32 bytes = 0;
+    for (u32 q = 0; q < 8; ++q) {
+      const bool have = q == 0 ? S.ps > 0 : (q == 1 ? (S.hs >= 1 && S.rs > 0) : q <= S.hs);
+      c->ns[q] = have ? T.alloc(S) : DT_NONE;
+      if (have) bytes += V ? 2u * NBY : NBY;
+    }
+    fence_proxy_async();
+    mbar_arrive_expect_tx(&c->lbar, bytes);
+    for (u32 q = 0; q < 8; ++q) {
+      if (c->ns[q] == DT_NONE) continue;
+      bulk_g2s(T.BK(c->ns[q]), H.gk + (size_t)q * K, NBY, &c->lbar);
+      if (V) bulk_g2s(T.BV(c->ns[q]), H.gv + (size_t)q * K, NBY, &c->lbar);
+    }
+    mbar_wait(&c->lbar, 0);
+    dt_plan<K, V>(T, S, n_ops, false);
+  }
+  __syncwarp();
+  const bool lt = (C.debug & 128u) != 0;
+  ull t0 = lt ? clock64() : 0, t1 = 0;
+  for (;;) {
+    if (*reinterpret_cast<volatile u32*>(&c->p_flags) == DT_NONE) break;
+    if (lt && lane == 0) { t1 = clock64(); c->tm[0] += t1 - t0; c->tm[5]++; }  // decisions (+ plan)
+    nbar_arrive(DT_BAR_READY, NB_);  // the groups run phase A of this slot
+    if (lane == 0) {
+      DtS* __restrict__ const Sp = &SS;
+    DtS& S = *Sp;
+      T.flush(S);  // helper requests of the decisions just taken and of the plan
+      // Alg.2 l.18-22: the old root keys are the first output of op i (TMA bulk store)
+      if (c->p_flags & F_NEW) {
+        const u32 n = c->p_out_n;
+        if (n) {
+          const u64 pos0 = (((u64)c->p_iop_hi << 32) | c->p_iop_lo) * (u64)K;
+          const u32 src = c->p_out_slot;
+          const bool bulk = (n & 3u) == 0 && ((reinterpret_cast<uintptr_t>(C.out_k + pos0) & 15u) == 0) &&
+                            (!V || !C.out_v || (reinterpret_cast<uintptr_t>(C.out_v + pos0) & 15u) == 0);
+          if (bulk) {
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            bulk_s2g(C.out_k + pos0, T.BK(src), n * 4u);
+            if (V && C.out_v) bulk_s2g(C.out_v + pos0, T.BV(src), n * 4u);
+            asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+          } else {
+            for (u32 q = 0; q < n; ++q) {
+              C.out_k[pos0 + q] = T.BK(src)[q];
+              if (V && C.out_v) C.out_v[pos0 + q] = T.BV(src)[q];
+            }
+          }
+        }
+      }
+    }
+    __syncwarp();
+    if (lt && lane == 0) { const ull t = clock64(); c->tm[2] += t - t1; t1 = t; }  // flush + output copy
+    nbar_sync(DT_BAR_DONE, NB_);  // phase A done, staged / refill data visible
+    if (lt && lane == 0) { t0 = clock64(); c->tm[1] += t0 - t1; }  // waiting for phase A
+    if (lane == 0) SS.stage = 0;
+    for (;;) {
+      if (lane == 0) {
+        DtS* __restrict__ const Sp = &SS;
+        DtS& S = *Sp;
+        c->njobs = 0;
+        bool done = false;
+        if (S.stage == 0) done = dt_fast<K, V>(T, S);
+        if (!done) done = dt_slow<K, V>(T, S, false);
+        if (done) dt_plan<K, V>(T, S, n_ops, false);
+        else c->p_flags = F_JOBS;
+        c->ctl_done = done ? 1u : 0u;
+      }
+      __syncwarp();
+      if (*reinterpret_cast<volatile u32*>(&c->ctl_done)) break;
+      nbar_arrive(DT_BAR_READY, NB_);  // the groups run the job list
+      nbar_sync(DT_BAR_DONE, NB_);
+    }
+  }
+  // ---- call end: the on-chip part back to the arena (a job list for the groups)
+  if (lane == 0) {
+    DtS* __restrict__ const Sp = &SS;
+    DtS& S = *Sp;
+    T.flush(S);
+    c->njobs = 0;
+    for (u32 q = 0; q < 8; ++q) {
+      const u32 sl = c->ns[q];
+      if (q >= 1) st_relaxed(T.stp(q), q <= S.hs ? ST_AVAIL : ST_EMPTY);
+      if (sl == DT_NONE) continue;
+      const u32 cnt = q == 0 ? S.ps : (q == 1 ? S.rs : K);
+      if (q > S.hs || cnt == 0) continue;
+      st_relaxed(&H.meta[q].kmin, T.BK(sl)[0]);
+      st_relaxed(&H.meta[q].kmax, T.BK(sl)[cnt - 1]);
+      T.job(J_STORE, q, sl);
+    }
+    c->p_flags = F_JOBS;
+  }
+  __syncwarp();
+  nbar_arrive(DT_BAR_READY, NB_);
+  nbar_sync(DT_BAR_DONE, NB_);
+  if (lane == 0) {
+    DtS* __restrict__ const Sp = &SS;
+    DtS& S = *Sp;
+    st_relaxed(H.hdr + H_HS, S.hs);
+    st_relaxed(H.hdr + H_RS, S.rs);
+    st_relaxed(H.hdr + H_PS, S.ps);
+    ull lin;
+    asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(lin) : "l"(H.hdr + H_LIN) : "memory");
+    asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(H.hdr + H_LIN), "l"(lin + n_ops) : "memory");
+    c->st[S_KEYS_OUT] += S.nout;
+    if (C.d_count && S.nout) atomicAdd(C.d_count, (ull)S.nout);
+    asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+    T.enqueue(RQ_END);
+    T.enqueue(RQ_STAGE, 0u, 0u, 0u, 0u, DT_NONE);
+    while (ld_acq_cta(&c->rq_done[0]) != c->rq_head[0] || ld_acq_cta(&c->rq_done[1]) != c->rq_head[1]) {}
+    ull* stat = reinterpret_cast<ull*>(H.hdr + H_STAT);
+    for (int q = 0; q < NSTAT; ++q)
+      if (c->st[q]) atomicAdd(stat + q, c->st[q]);
+    if (lt) {
+      ull* tms = reinterpret_cast<ull*>(H.hdr + H_TIME);
+      for (int q = 0; q < 12; ++q) { atomicAdd(tms + 16 + q, c->tm[q]); atomicAdd(tms + q, c->ts[q]); }
+    }
+    c->p_flags = DT_NONE;
+  }
+  __syncwarp();
+  nbar_arrive(DT_BAR_READY, NB_);  // the groups leave
 }
 
 // =========================================================================================
@@ -1361,12 +1593,18 @@ __global__ void __launch_bounds__(DT_BLOCK, 1) bgpq_dtop_kernel(HeapArgs H, Call
       asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     __syncthreads();
-    if (threadIdx.x >= DT_NTC) {
-      if (threadIdx.x == DT_NTC) dt_helper<K, V>(T, 0u);
-      if (threadIdx.x == DT_NTC + 32) dt_helper<K, V>(T, 1u);
+    const bool ctlw = (C.debug & 512u) != 0;  // test switch 512: the control-warp driver (dt_control)
+    if (threadIdx.x >= DT_NTC + 32) {
+      if (threadIdx.x == DT_NTC + 32) dt_helper<K, V>(T, 0u);
+      if (threadIdx.x == DT_NTC + 64) dt_helper<K, V>(T, 1u);
       return;
     }
-    dt_top<K, V>(T);
+    if (threadIdx.x >= DT_NTC) {
+      if (ctlw) dt_control<K, V>(T);
+      return;
+    }
+    if (ctlw) dt_groups2<K, V>(T);
+    else dt_top<K, V>(T);
     return;
   }
   // ---- walkers

@@ -20,7 +20,7 @@ e[0].record(); q.deletemin(n, out); e[1].record(); torch.cuda.synchronize()
 d = raw() - t1
 slots = max(d[21], 1)
 print("del ms %.2f us/op %.2f slots %d conflicts %d" % (e[0].elapsed_time(e[1]), e[0].elapsed_time(e[1]) * 1e3 / (n // K), d[21], d[22]))
-for i, nm in enumerate(["plan", "phaseA", "G2 stage wait", "refill wait", "phaseB"]):
+for i, nm in enumerate(["plan/decisions", "phaseA(wait)", "G2 wait|flush", "data waits", "phaseB"]):
     print("  %-14s %8.0f cyc/slot" % (nm, d[16 + i] / slots))
 print("  helper lock wait %8.0f cyc/slot" % (d[23] / slots))
 print("  G0 out+merge %8.0f  G1 merge %8.0f  G2 wait+merge %8.0f  rounds/slot %.2f" % (d[24] / slots, d[25] / slots, d[26] / slots, d[27] / slots))
