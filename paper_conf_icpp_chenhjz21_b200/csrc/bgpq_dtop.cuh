@@ -185,6 +185,16 @@ __device__ __forceinline__ void grp_bar(int g) {
 template <int K, bool V>
 __device__ __forceinline__ void grp_split(int t, const u32* zk, const u32* zv, int na, const u32* wk, const u32* wv,
                                           int nb, int ma, u32* xk, u32* xv, u32* yk, u32* yv, bool win = false) {
+#ifndef BGPQ_NO_BITONIC
+  if constexpr (!V) {  // keys only, full batches: the search-free bitonic split (bgpq_prim.cuh)
+    constexpr int NB = K < DT_GT ? K : DT_GT;
+    if (!win && na == K && nb == K && ma == K) {
+      // named barrier 8 + group: its own id (grp_bar uses 2 + g with all DT_GT threads)
+      if (t < NB) bitonic_split_full<K, NB, false>(t, 8 + (int)(threadIdx.x / DT_GT), zk, zv, wk, wv, xk, xv, yk, yv);
+      return;
+    }
+  }
+#endif
   if (!win) {
     constexpr int NW = (2 * K / 32 < DT_GT / 32) ? 2 * K / 32 : DT_GT / 32;
     grp_merge_warp<K, NW, V>(t >> 5, zk, zv, na, wk, wv, nb, ma, xk, xv, yk, yv);

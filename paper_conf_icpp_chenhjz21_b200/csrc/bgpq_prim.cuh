@@ -585,13 +585,167 @@ __device__ __forceinline__ void cta_merge_warp(const u32* __restrict__ zk, const
   grp_merge_warp<KMAX, NW, V>((int)(threadIdx.x >> 5), zk, zv, na, wk, wv, nb, ma, xk, xv, yk, yv);
 }
 
+// ----------------------------------------------------------------------------------------
+// SORT_SPLIT of two full sorted K-batches (Na = Nb = Ma = K, the common case of P:196) without
+// co-rank searches (v5): X = K smallest, Y = K largest.  min / max of Z[p] and W[K-1-p]
+// (Batcher's half-cleaner on Z ++ reverse(W)) put exactly the K smallest into L and the rest
+// into U, each a bitonic sequence; each half is then sorted by a bitonic merge — strides below
+// E = 2K/NT inside a thread's registers, strides up to 31 threads with __shfl_xor_sync, larger
+// ones through the output tile in shared memory.  Threads 0..NT/2-1 build X, the rest Y; thread
+// u of a half owns positions [u*E, u*E+E).  With values the comparison key is the stable
+// composite (key, Z before W, index), so the result equals the stable merge's order; keys only
+// compares the 32-bit keys.  bar_id / NT: the named barrier of the NT participating threads.
+// ----------------------------------------------------------------------------------------
+template <int K, int NT, bool V>
+__device__ __forceinline__ void bitonic_split_full(const int t, const int bar_id, const u32* __restrict__ zk,
+                                                   const u32* __restrict__ zv, const u32* __restrict__ wk,
+                                                   const u32* __restrict__ wv, u32* __restrict__ xk,
+                                                   u32* __restrict__ xv, u32* __restrict__ yk, u32* __restrict__ yv) {
+  constexpr int HT = NT / 2;   // threads per half
+  constexpr int E = K / HT;    // elements per thread
+  static_assert(E >= 1 && (E & (E - 1)) == 0 && E * HT == K, "K must be a multiple of NT/2 (power of two)");
+  using T = typename std::conditional<V, u64, u32>::type;
+  const int half = t / HT, u = t % HT;
+  u32* ok = half ? yk : xk;
+  u32* ov = half ? yv : xv;
+  T c[E];
+  // 1. half-cleaner, strided layout: c[e] holds position p = e*HT + u of the half
+#pragma unroll
+  for (int e = 0; e < E; ++e) {
+    const int p = e * HT + u, q = K - 1 - p;
+    T a, b;
+    if constexpr (V) {
+      a = ((u64)zk[p] << 32) | (u32)p;
+      b = ((u64)wk[q] << 32) | 0x80000000u | (u32)q;
+    } else {
+      a = zk[p];
+      b = wk[q];
+    }
+    c[e] = half ? (a < b ? b : a) : (a < b ? a : b);
+  }
+  // 2. bitonic merge strides j >= HT: register index bits (strided layout)
+#pragma unroll
+  for (int jr = E / 2; jr >= 1; jr >>= 1) {
+#pragma unroll
+    for (int e = 0; e < E; ++e) {
+      if ((e & jr) == 0) {
+        const T a = c[e], b = c[e + jr];
+        c[e] = a < b ? a : b;
+        c[e + jr] = a < b ? b : a;
+      }
+    }
+  }
+  // 3. transpose through the output tile to the blocked layout: c[e] = position u*E + e
+#pragma unroll
+  for (int e = 0; e < E; ++e) {
+    ok[e * HT + u] = V ? (u32)(c[e] >> 32) : (u32)c[e];
+    if constexpr (V) ov[e * HT + u] = (u32)c[e];
+  }
+  asm volatile("bar.sync %0, %1;" ::"r"(bar_id), "n"(NT) : "memory");
+#pragma unroll
+  for (int e = 0; e < E; ++e) {
+    if constexpr (V) c[e] = ((u64)ok[u * E + e] << 32) | ov[u * E + e];
+    else c[e] = ok[u * E + e];
+  }
+  asm volatile("bar.sync %0, %1;" ::"r"(bar_id), "n"(NT) : "memory");
+  // 4. strides HT/2 .. E: across threads (distance j/E), then < E inside the thread
+#pragma unroll
+  for (int j = HT / 2; j >= 1; j >>= 1) {
+    if (j >= E) {
+      const int d = j / E;
+      const bool upper = (u & d) != 0;
+      if (d < 32) {
+#pragma unroll
+        for (int e = 0; e < E; ++e) {
+          T pv;
+          if constexpr (V) {
+            const u32 lo = __shfl_xor_sync(0xffffffffu, (u32)c[e], d);
+            const u32 hi = __shfl_xor_sync(0xffffffffu, (u32)(c[e] >> 32), d);
+            pv = ((u64)hi << 32) | lo;
+          } else {
+            pv = __shfl_xor_sync(0xffffffffu, c[e], d);
+          }
+          c[e] = upper ? (c[e] > pv ? c[e] : pv) : (c[e] < pv ? c[e] : pv);
+        }
+      } else {  // across warps: exchange through the tile
+        const int p0 = u * E, pp0 = (u ^ d) * E;
+#pragma unroll
+        for (int e = 0; e < E; ++e) {
+          ok[p0 + e] = V ? (u32)(c[e] >> 32) : (u32)c[e];
+          if constexpr (V) ov[p0 + e] = (u32)c[e];
+        }
+        asm volatile("bar.sync %0, %1;" ::"r"(bar_id), "n"(NT) : "memory");
+        T pv[E];
+#pragma unroll
+        for (int e = 0; e < E; ++e) {
+          if constexpr (V) pv[e] = ((u64)ok[pp0 + e] << 32) | ov[pp0 + e];
+          else pv[e] = ok[pp0 + e];
+        }
+        asm volatile("bar.sync %0, %1;" ::"r"(bar_id), "n"(NT) : "memory");
+#pragma unroll
+        for (int e = 0; e < E; ++e) c[e] = upper ? (c[e] > pv[e] ? c[e] : pv[e]) : (c[e] < pv[e] ? c[e] : pv[e]);
+      }
+    }
+  }
+#pragma unroll
+  for (int jr = E / 2; jr >= 1; jr >>= 1) {
+#pragma unroll
+    for (int e = 0; e < E; ++e) {
+      if ((e & jr) == 0) {
+        const T a = c[e], b = c[e + jr];
+        c[e] = a < b ? a : b;
+        c[e + jr] = a < b ? b : a;
+      }
+    }
+  }
+  // 5. write back, blocked (values gathered from the source index)
+  const int p0 = u * E;
+  if constexpr (V) {
+    u32 kk[E], vv[E];
+#pragma unroll
+    for (int e = 0; e < E; ++e) {
+      const u32 lw = (u32)c[e];
+      const u32 idx = lw & 0x7FFFFFFFu;
+      kk[e] = (u32)(c[e] >> 32);
+      vv[e] = (lw & 0x80000000u) ? wv[idx] : zv[idx];
+    }
+#pragma unroll
+    for (int e = 0; e < E; ++e) { ok[p0 + e] = kk[e]; ov[p0 + e] = vv[e]; }
+  } else {
+    if constexpr (E % 4 == 0) {
+#pragma unroll
+      for (int e = 0; e < E; e += 4)
+        *reinterpret_cast<uint4*>(ok + p0 + e) = make_uint4(c[e], c[e + 1], c[e + 2], c[e + 3]);
+    } else {
+#pragma unroll
+      for (int e = 0; e < E; ++e) ok[p0 + e] = c[e];
+    }
+  }
+}
+
 // The SORT_SPLIT used on the hot path: register-window merge path with VT = 4 outputs per
 // thread (threads 0 .. 2K/4-1 of the NT compute threads take part).  Measured on B200
 // (tools/micro_merge.cu, K = 1024, NT = 512): 1540 cycles keys-only / 2110 key+value, vs
 // 2110 / 2190 for the co-ranking merge.
+// Keys-only splits of two full K-batches use the search-free bitonic split (920 vs 1540 cycles
+// at K = 1024, micro_merge.txt) on the first min(512, K) threads with named barrier 5; the
+// caller's CTA barrier after the split joins the rest.
+constexpr int BAR_BITONIC = 5;
 template <int K, int NT, bool V>
 __device__ __forceinline__ void sort_split(const u32* zk, const u32* zv, int na, const u32* wk, const u32* wv,
                                            int nb, int ma, u32* xk, u32* xv, u32* yk, u32* yv) {
+#ifndef BGPQ_NO_BITONIC
+  if constexpr (!V) {
+    constexpr int NB = (K < 512 ? K : 512) <= NT ? (K < 512 ? K : 512) : 0;
+    if constexpr (NB >= 64) {
+      if (na == K && nb == K && ma == K) {
+        if ((int)threadIdx.x < NB)
+          bitonic_split_full<K, NB, false>((int)threadIdx.x, BAR_BITONIC, zk, zv, wk, wv, xk, xv, yk, yv);
+        return;
+      }
+    }
+  }
+#endif
   constexpr int NTM = (2 * K / 4 <= NT) ? 2 * K / 4 : NT;
   cta_merge_win<K, NTM, V>(zk, zv, na, wk, wv, nb, ma, xk, xv, yk, yv);
 }

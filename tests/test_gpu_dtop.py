@@ -131,3 +131,25 @@ def test_stats_count_every_level():
     # 1024 nodes: a walk has at most log2(1024) = 10 levels and almost every op goes deep
     assert 5 * (n // K) < d["del_levels"] <= 10 * (n // K)
     q.close()
+
+
+def test_reused_heap_full_size_multiset():
+    """C2 size, heap reused across drains (|root| = 0 state): after every INSERT call the keys
+    stored in the heap (root, pBuffer, nodes 2..heapSize) are exactly the input multiset, and the
+    drain returns sorted(input).  Guards the insert pipeline's write-back ordering, which the
+    structural invariants alone cannot see (a lost key leaves a valid heap)."""
+    n, K = 1 << 27, 1024
+    keys = synth.keys(n, seed=synth.SEEDS["C2"])
+    srt = np.sort(keys)
+    q = pkg.BGPQ(capacity=n, K=K, values=False)
+    dk = _dev(keys)
+    for rep in range(2):
+        q.insert(dk)
+        nk, _, _, h = q.dump()
+        hs, rs, ps = h["heapSize"], h["rootSize"], h["pbSize"]
+        nk2 = nk.reshape(-1, K)
+        parts = [nk2[1, :rs], nk2[0, :ps]] + ([nk2[2:hs + 1].ravel()] if hs >= 2 else [])
+        assert np.array_equal(np.sort(np.concatenate(parts)), srt), rep
+        ok, _ = q.deletemin(n)
+        assert np.array_equal(_host(ok), srt), rep
+    q.close()

@@ -1,7 +1,7 @@
 #!/bin/bash
 # Round-end evidence for the current build (run under gpurun)
 cd "$GRAFT_REPO_ROOT"; mkdir -p gpurun_out
-timeout 1200 python -m pytest tests -m gpu -x -q > gpurun_out/pytest_gpu.log 2>&1; echo "pytest rc=$?" >> gpurun_out/pytest_gpu.log; tail -2 gpurun_out/pytest_gpu.log
+timeout -s KILL 1200 python -m pytest tests -m gpu -x -q > gpurun_out/pytest_gpu.log 2>&1; echo "pytest rc=$?" >> gpurun_out/pytest_gpu.log; tail -2 gpurun_out/pytest_gpu.log
 timeout 900 python bench.py --steps 5 --warmup 3 > gpurun_out/bench_w4.log 2>&1; echo "bench rc=$?"
 timeout 900 python bench.py --steps 3 --warmup 3 --values --no-cpu-baseline > gpurun_out/bench_w8.log 2>&1; echo "bench w8 rc=$?"
 timeout 900 python bench.py --impl reference --steps 2 --warmup 3 > gpurun_out/bench_ref.log 2>&1; echo "ref rc=$?"

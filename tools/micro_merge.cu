@@ -27,6 +27,7 @@ __global__ void k_merge(const u32* in, const int* sizes, u32* out, long long* cy
     else if constexpr (MODE == 1) cta_path_merge<K, NT, V>(z, zv, na, w, wv, nb, ma, x, xv, y, yv);
     else if constexpr (MODE == 2) cta_merge_win<K, NTM, V>(z, zv, na, w, wv, nb, ma, x, xv, y, yv);
     else if constexpr (MODE == 3) cta_merge_warp<K, NTM, V>(z, zv, na, w, wv, nb, ma, x, xv, y, yv);
+    else if constexpr (MODE == 7) bitonic_split_full<K, NTM, V>(threadIdx.x, 1, z, zv, w, wv, x, xv, y, yv);
     else if constexpr (MODE == 4) { if (threadIdx.x == 0) x[r & 1023] = r; }
     else if constexpr (MODE == 5) { const int c = warp_corank(z, na, w, nb, (threadIdx.x >> 5) * 128); if ((threadIdx.x & 31) == 0) x[threadIdx.x >> 5] = c; }
     else if constexpr (MODE == 6) {
@@ -59,6 +60,7 @@ bool run(const char* name, u32* d_in, int* d_sz, u32* d_out, long long* d_cyc, b
     if (!timing && tcase % 7 == 0) na = K;
     if (!timing && tcase % 5 == 0) nb = K;
     int ma = timing ? K : (int)(nxt() % (na + nb + 1));
+    if (MODE == 7) { na = nb = ma = K; }
     if (!timing && tcase % 3 == 0) ma = std::min(K, na + nb);
     if (ma > K || na + nb - ma > K) { ma = std::min(K, na + nb); if (na + nb - ma > K) continue; }
     const u32 mod = (tcase % 4 == 0) ? 16u : 0xFFFFFFFFu;
@@ -118,6 +120,11 @@ int main() {
     ok &= run<512, 256, 2, false>("merge_win NTM=256 keys", d_in, d_sz, d_out, d_cyc, timing);
     ok &= run<512, 128, 2, false>("merge_win NTM=128 keys", d_in, d_sz, d_out, d_cyc, timing);
     ok &= run<1024, 1024, 2, false>("merge_win NTM=1024 keys", d_in, d_sz, d_out, d_cyc, timing);
+    ok &= run<512, 512, 7, false>("bitonic_full NT=512 keys", d_in, d_sz, d_out, d_cyc, timing);
+    ok &= run<256, 256, 7, false>("bitonic_full NT=256 keys", d_in, d_sz, d_out, d_cyc, timing);
+    ok &= run<128, 128, 7, false>("bitonic_full NT=128 keys", d_in, d_sz, d_out, d_cyc, timing);
+    ok &= run<512, 512, 7, true>("bitonic_full NT=512 key+val", d_in, d_sz, d_out, d_cyc, timing);
+    ok &= run<256, 256, 7, true>("bitonic_full NT=256 key+val", d_in, d_sz, d_out, d_cyc, timing);
     ok &= run<512, 4, 3, false>("merge_warp NW=4 keys", d_in, d_sz, d_out, d_cyc, timing);
     ok &= run<512, 8, 3, false>("merge_warp NW=8 keys", d_in, d_sz, d_out, d_cyc, timing);
     ok &= run<512, 16, 3, false>("merge_warp NW=16 keys", d_in, d_sz, d_out, d_cyc, timing);
