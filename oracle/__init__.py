@@ -7,7 +7,7 @@ Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s ``cpu_baseline``
 Everything here is a thin ctypes marshalling layer over ``bgpq_oracle.cpp`` (plain C++17,
 see its header for what each function transcribes from PAPER.md), plus ``build()``.
 
-Pins: see tests/test_oracle_*.py.  Parity status per function is in DESIGN.md §Oracle.
+Pins: see tests/test_oracle.py.  Parity status per function is in DESIGN.md §Oracle.
 """
 from __future__ import annotations
 

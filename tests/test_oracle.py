@@ -303,3 +303,41 @@ def test_invariant_checker_catches_corruption():
     bad_st = st.copy(); bad_st[h["heapSize"] + 1] = oracle.AVAIL    # AVAIL beyond heapSize
     assert oracle.check_invariants(*args, nk, bad_st)[0] == -3
     assert oracle.check_invariants(K, q.cap, h["heapSize"], K + 1, 0, nk, st)[0] == -1
+
+
+@pytest.mark.parametrize("K", [4, 64])
+def test_seq_model_sorted_input_special_cases(K):
+    """Special cases fixed by Alg.1 and SORT_SPLIT's definition.
+
+    Ascending full-K batches: every new batch is >= every stored key, so the root section
+    and each INSERT_HEAPIFY level keep their node (no-op split) and batch j lands whole at
+    node tar = j+1 (heapSize++ per op, Alg.1 l.16-18): the node array is the input in BFS
+    order.  Descending batches: every batch is <= every stored key, so every split along
+    the path is a pure swap and the root always holds the last batch.
+    """
+    nb = 37                                     # ragged last level of the tree
+    base = np.sort(synth.keys(nb * K, seed=5))
+    q = oracle.SeqBGPQ(K, nb + 2)
+    for j in range(nb):
+        q.insert(base[j * K:(j + 1) * K])
+    nk, _, st = q.dump()
+    for j in range(nb):
+        assert np.array_equal(nk[j + 1], base[j * K:(j + 1) * K]), j
+        assert st[j + 1] == oracle.AVAIL
+    c = q.counters()
+    assert c["ins_swap"] == 0 and c["ins_merge"] == 0
+    assert c["ins_noop"] == c["ins_levels"]
+    assert _check_inv(q) == (0, 0)
+
+    desc = base[::-1].copy()
+    q = oracle.SeqBGPQ(K, nb + 2)
+    for j in range(nb):
+        q.insert(desc[j * K:(j + 1) * K])
+    nk, _, _ = q.dump()
+    assert np.array_equal(nk[1], np.sort(desc[(nb - 1) * K:]))
+    c = q.counters()
+    assert c["ins_noop"] == 0 and c["ins_merge"] == 0
+    assert c["ins_swap"] == c["ins_levels"]
+    assert _check_inv(q) == (0, 0)
+    out = np.concatenate([q.deletemin(K)[0] for _ in range(nb)])
+    assert np.array_equal(out, base)
