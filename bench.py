@@ -192,6 +192,117 @@ def cpu_baseline(args):
                       f"std::multiset oracle, 1 pinned host core, {dt:.1f} s"}
 
 
+def run_mix(args, world, rank, local):
+    """C2 mix: prefill 2^prefill keys (stream 22), then
+    bgpq_run_mixed over n/K insert(K) + n/K deletemin(K) ops interleaved as pairs.
+    keys/s = (keys inserted + keys deleted) / 2 / t.  Each step re-builds the
+    prefilled heap untimed (drain + prefill insert), then times the mixed call only."""
+    import torch
+    import synth
+    import paper_conf_icpp_chenhjz21_b200 as pkg
+
+    torch.cuda.set_device(local)
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    n, K, P = 1 << args.n_log2, args.K, 1 << args.prefill_log2
+    w = 8 if args.values else 4
+    n_pairs = n // K
+    types, sizes = synth.mixed_ops(n_pairs, K, seed=synth.SEEDS["C2_mix"])
+    in_off = np.zeros(2 * n_pairs, np.uint64)
+    in_off[0::2] = np.arange(n_pairs, dtype=np.uint64) * K
+    keys = synth.keys(n, seed=synth.SEEDS["C2"] + rank, dist=args.dist)
+    pre = synth.keys(P, seed=synth.SEEDS["C2_mix"] + rank, dist=args.dist)
+    d_types = torch.from_numpy(types).cuda()
+    d_sizes = torch.from_numpy(sizes.view(np.int32)).cuda()
+    d_off = torch.from_numpy(in_off.view(np.int64)).cuda()
+    dk = torch.from_numpy(keys.view(np.int32)).cuda()
+    dpre = torch.from_numpy(pre.view(np.int32)).cuda()
+    dv = torch.arange(n, dtype=torch.int32, device="cuda") if args.values else None
+    dpv = torch.arange(P, dtype=torch.int32, device="cuda") if args.values else None
+    out_k = torch.empty(2 * n_pairs * K, dtype=torch.int32, device="cuda")
+    out_v = torch.empty(2 * n_pairs * K, dtype=torch.int32, device="cuda") if args.values else None
+    cnt = torch.zeros(2 * n_pairs, dtype=torch.int32, device="cuda")
+    drain = torch.empty(n + P, dtype=torch.int32, device="cuda")
+    drain_v = torch.empty(n + P, dtype=torch.int32, device="cuda") if args.values else None
+    q = pkg.BGPQ(capacity=n + P + K, K=K, values=args.values)
+    stream = torch.cuda.current_stream()
+
+    def reset():
+        sz = q.size(stream=stream)
+        if sz:
+            q.deletemin(sz, drain, drain_v, stream=stream)
+        q.insert(dpre, dpv, stream=stream)
+
+    def mixed():
+        q.run_mixed(d_types, d_sizes, d_off, dk, dv, out_k, out_v, cnt, None, stream=stream)
+
+    for _ in range(args.warmup):
+        reset(); mixed()
+    torch.cuda.synchronize()
+    # parity of the last warm-up step at full size: every deletemin returned K keys, and the
+    # key multiset is conserved (mix outputs + drain == prefill + inserted keys)
+    assert q.size(stream=stream) == P
+    q.deletemin(P, drain, drain_v, stream=stream)
+    torch.cuda.synchronize()
+    mask = 0xFFFFFFFF
+    got = torch.cat([out_k.view(2 * n_pairs, K)[1::2].reshape(-1), drain[:P]]).to(torch.int64) & mask
+    want = torch.cat([dk, dpre]).to(torch.int64) & mask
+    ok_parity = bool((cnt[1::2] == K).all().item()) and bool(torch.equal(torch.sort(got)[0], torch.sort(want)[0]))
+    del got, want
+
+    ms, launches, acc = [], 0, None
+    clk = ClockSampler(local)
+    clk.start()
+    for _ in range(args.steps):
+        reset()
+        st0 = q.stats()  # synchronizes; counters bracket the mixed call only
+        l0 = pkg.launch_count()
+        e0 = torch.cuda.Event(enable_timing=True); e1 = torch.cuda.Event(enable_timing=True)
+        if dist: dist.barrier()
+        torch.cuda.synchronize()
+        e0.record(stream); mixed(); e1.record(stream)
+        torch.cuda.synchronize()
+        ms.append(e0.elapsed_time(e1))
+        launches += pkg.launch_count() - l0
+        st1 = q.stats()
+        d = {k: st1[k] - st0[k] for k in st1}
+        acc = d if acc is None else {k: acc[k] + d[k] for k in d}
+    clocks = clk.stop()
+    total_ms = max_over_ranks(float(np.sum(ms)), dist, device="cuda")
+    ms_per_step = total_ms / args.steps
+    value = job_throughput(n, args.steps, world, total_ms)
+    dst = {k: v // args.steps for k, v in acc.items()}
+    bm = byte_model(dst, K, w)
+    peak, peak_src = _peaks()
+    achieved = bm["total"] / (ms_per_step / 1e3) / 1e9
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": "keys/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+            "config": {"workload": (f"C2 mix: prefill 2^{args.prefill_log2} then {n_pairs} insert(K) + "
+                                    f"{n_pairs} deletemin(K) ops as pairs, 2^{args.n_log2} {args.dist} "
+                                    f"keys, K={K}, w={w} B; keys/s = (in + out)/2/t"),
+                       "n_keys": n, "K": K, "w_bytes": w, "prefill": P, "dist": args.dist,
+                       "execution": "bgpq_run_mixed: persistent CTAs, per-node locks + lock warp",
+                       "l2": "heap and inputs larger than the 126 MB L2; no flush"},
+            "parallelism": "replicas only (one linearizable heap per GPU)",
+            "roofline": {"bound": "hbm", "kernel": "bgpq_run_mixed kernel", "achieved": achieved,
+                         "peak": peak, "unit": "GB/s", "frac": achieved / peak, "traffic": None,
+                         "peak_source": peak_src, "alg_bytes_per_launch": bm["total"]},
+            "counters_per_step": dst,
+            "gpu_launches": launches,
+            "clocks": clocks,
+            "e2e": None,
+            "parity_warmup_multiset_conserved": ok_parity,
+        }
+        print(json.dumps(line), flush=True)
+    if dist:
+        dist.destroy_process_group()
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -206,6 +317,10 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--profile-steps", type=int, default=0, help="ncu mode: run N untimed steps and exit")
+    ap.add_argument("--mix", action="store_true",
+                    help="C2 50/50 concurrent mix (paper E4 shape, P:428): prefill, then insert(K)/deletemin(K) "
+                         "pairs on the persistent CTAs (bgpq_run_mixed)")
+    ap.add_argument("--prefill-log2", type=int, default=23)
     ap.add_argument("--mode", default="locks", choices=["locks", "server"],
                     help="execution: default (insert level pipeline + deletemin top CTA with walkers "
                          "taking the paper's per-node locks), or the root-server CTA")
@@ -214,6 +329,9 @@ def main():
 
     if args.impl == "reference":
         run_reference(args, world, rank)
+        return
+    if args.mix:
+        run_mix(args, world, rank, local)
         return
 
     import torch
