@@ -1,7 +1,10 @@
-"""Summarise an ncu --set full report into JSON: python tools/ncu_summary.py rep.ncu-rep out.json"""
+"""Summarise an ncu --set full report into JSON: python tools/ncu_summary.py rep.ncu-rep|raw.csv out.json"""
 import csv, json, subprocess, sys
 rep, out = sys.argv[1], sys.argv[2]
-txt = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+if rep.endswith(".csv"):  # already exported with `ncu -i rep --page raw --csv` (tools/ncu_export.sh)
+    txt = open(rep).read()
+else:
+    txt = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
 rows = list(csv.reader(txt.splitlines()))
 h, units, v = rows[0], rows[1], rows[2]
 keep = ["Kernel Name", "gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum",
