@@ -227,6 +227,8 @@ def run_mix(args, world, rank, local):
     drain = torch.empty(n + P, dtype=torch.int32, device="cuda")
     drain_v = torch.empty(n + P, dtype=torch.int32, device="cuda") if args.values else None
     q = pkg.BGPQ(capacity=n + P + K, K=K, values=args.values)
+    if args.grid:
+        q.set_grid(args.grid)
     stream = torch.cuda.current_stream()
 
     def reset():
@@ -287,6 +289,7 @@ def run_mix(args, world, rank, local):
                                     f"keys, K={K}, w={w} B; keys/s = (in + out)/2/t"),
                        "n_keys": n, "K": K, "w_bytes": w, "prefill": P, "dist": args.dist,
                        "execution": "bgpq_run_mixed: persistent CTAs, per-node locks + lock warp",
+                       "grid": q.grid(),
                        "l2": "heap and inputs larger than the 126 MB L2; no flush"},
             "parallelism": "replicas only (one linearizable heap per GPU)",
             "roofline": {"bound": "hbm", "kernel": "bgpq_run_mixed kernel", "achieved": achieved,
@@ -321,6 +324,7 @@ def main():
                     help="C2 50/50 concurrent mix (paper E4 shape, P:428): prefill, then insert(K)/deletemin(K) "
                          "pairs on the persistent CTAs (bgpq_run_mixed)")
     ap.add_argument("--prefill-log2", type=int, default=23)
+    ap.add_argument("--grid", type=int, default=0, help="--mix: persistent CTAs of the mixed call (0 = all co-resident)")
     ap.add_argument("--mode", default="locks", choices=["locks", "server"],
                     help="execution: default (insert level pipeline + deletemin top CTA with walkers "
                          "taking the paper's per-node locks), or the root-server CTA")
