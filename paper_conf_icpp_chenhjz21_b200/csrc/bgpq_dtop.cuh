@@ -186,7 +186,7 @@ template <int K, bool V>
 __device__ __forceinline__ void grp_split(int t, const u32* zk, const u32* zv, int na, const u32* wk, const u32* wv,
                                           int nb, int ma, u32* xk, u32* xv, u32* yk, u32* yv, bool win = false) {
 #ifndef BGPQ_NO_BITONIC
-  if constexpr (!V) {  // keys only, full batches: the search-free bitonic split (bgpq_prim.cuh)
+  if constexpr (!V && K >= BITONIC_MIN_K) {  // keys only, full batches: bitonic split (bgpq_prim.cuh)
     constexpr int NB = K < DT_GT ? K : DT_GT;
     if (!win && na == K && nb == K && ma == K) {
       // named barrier 8 + group: its own id (grp_bar uses 2 + g with all DT_GT threads)

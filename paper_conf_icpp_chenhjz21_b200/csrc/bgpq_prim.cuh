@@ -729,15 +729,18 @@ __device__ __forceinline__ void bitonic_split_full(const int t, const int bar_id
 // 2110 / 2190 for the co-ranking merge.
 // Keys-only splits of two full K-batches use the search-free bitonic split (920 vs 1540 cycles
 // at K = 1024, micro_merge.txt) on the first min(512, K) threads with named barrier 5; the
-// caller's CTA barrier after the split joins the rest.
+// caller's CTA barrier after the split joins the rest.  Only at K >= 512: below it the
+// bitonic network's per-stage named barriers cost more than the merge path saves (C3 sweep,
+// profiles/r1/final2_sweep_c3.jsonl vs c3_gate.jsonl: K = 128 / 256 inserts 10-12 % faster without it).
 constexpr int BAR_BITONIC = 5;
+constexpr int BITONIC_MIN_K = 512;
 template <int K, int NT, bool V>
 __device__ __forceinline__ void sort_split(const u32* zk, const u32* zv, int na, const u32* wk, const u32* wv,
                                            int nb, int ma, u32* xk, u32* xv, u32* yk, u32* yv) {
 #ifndef BGPQ_NO_BITONIC
   if constexpr (!V) {
     constexpr int NB = (K < 512 ? K : 512) <= NT ? (K < 512 ? K : 512) : 0;
-    if constexpr (NB >= 64) {
+    if constexpr (NB >= 64 && K >= BITONIC_MIN_K) {
       if (na == K && nb == K && ma == K) {
         if ((int)threadIdx.x < NB)
           bitonic_split_full<K, NB, false>((int)threadIdx.x, BAR_BITONIC, zk, zv, wk, wv, xk, xv, yk, yv);
