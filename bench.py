@@ -165,9 +165,9 @@ def _config(args):
                          f"then deletemin all, K={args.K}, {'key+value' if args.values else 'keys only'} "
                          f"(w={w} B)"),
             "n_keys": 1 << args.n_log2, "K": args.K, "w_bytes": w, "dist": args.dist,
-            "execution": ({"insert": "level pipeline (bgpq_ins_pipe_kernel, one CTA per heap level)",
-                           "deletemin": "top CTA + walker CTAs (bgpq_dtop_kernel)"} if args.mode == "locks" else
-                          {"insert": "root-server (bgpq_srv_kernel)", "deletemin": "root-server (bgpq_srv_kernel)"}),
+            "execution": ({"insert": "level pipeline (bgpq_ins_pipe2_kernel, one CTA per heap level)",
+                           "deletemin": "top CTA + walker CTAs (bgpq_dtop_kernel)"} if args.mode == "default" else
+                          {"insert": "per-node locks (bgpq_locks_kernel)", "deletemin": "per-node locks (bgpq_locks_kernel)"}),
             "l2": f"inputs and heap ({(1 << args.n_log2) * w * 3 >> 20} MiB) "
                                           "larger than the 126 MB L2; no flush"}
 
@@ -325,9 +325,10 @@ def main():
                          "pairs on the persistent CTAs (bgpq_run_mixed)")
     ap.add_argument("--prefill-log2", type=int, default=23)
     ap.add_argument("--grid", type=int, default=0, help="--mix: persistent CTAs of the mixed call (0 = all co-resident)")
-    ap.add_argument("--mode", default="locks", choices=["locks", "server"],
+    ap.add_argument("--mode", default="default", choices=["default", "locks"],
                     help="execution: default (insert level pipeline + deletemin top CTA with walkers "
-                         "taking the paper's per-node locks), or the root-server CTA")
+                         "taking the paper's per-node locks), or the paper-literal per-node-lock engine "
+                         "for every call (BGPQ_FLAG_LOCKS)")
     args = ap.parse_args()
     world, rank, local = _dist_setup()
 
@@ -355,7 +356,7 @@ def main():
     dv = torch.arange(n, dtype=torch.int32, device="cuda") if args.values else None
     out_k = torch.empty(n, dtype=torch.int32, device="cuda")
     out_v = torch.empty(n, dtype=torch.int32, device="cuda") if args.values else None
-    q = pkg.BGPQ(capacity=n, K=K, values=args.values, server=(args.mode == "server"))
+    q = pkg.BGPQ(capacity=n, K=K, values=args.values, locks=(args.mode == "locks"))
     stream = torch.cuda.current_stream()
 
     def step(ev=None):
@@ -453,7 +454,7 @@ def main():
             "config": _config(args),
             "parallelism": "replicas only (one linearizable heap per GPU)",
             "phases_ms": {"insert": float(np.mean(ins_ms)), "deletemin": float(np.mean(del_ms))},
-            "roofline": {"bound": "hbm", "kernel": ("bgpq_dtop_kernel (DELETEMIN launch)" if args.mode == "locks" else "bgpq_srv_kernel (DELETEMIN launch)"),
+            "roofline": {"bound": "hbm", "kernel": ("bgpq_dtop_kernel (DELETEMIN launch)" if args.mode == "default" else "bgpq_locks_kernel (DELETEMIN launch)"),
                          "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
                          "traffic": traffic, "peak_source": peak_src,
                          "alg_bytes_per_launch": bm["deletemin"]},

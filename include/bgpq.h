@@ -47,11 +47,8 @@ enum {
   BGPQ_FLAG_VALUES = 1u, /* store a uint32 value with every key (w = 8 B per entry)        */
   BGPQ_FLAG_SERIAL = 2u, /* execute operations one at a time on a single CTA (test mode:
                             the node layout then equals the sequential Alg.1-3 model)     */
-  BGPQ_FLAG_LOCKS = 4u,  /* per-node-lock execution of every call (the mixed-call engine,
+  BGPQ_FLAG_LOCKS = 4u   /* per-node-lock execution of every call (the mixed-call engine,
                             used for insert-only and deletemin-only calls too)              */
-  BGPQ_FLAG_SERVER = 8u  /* root-server execution: one CTA holds the root, the pBuffer and
-                            the top levels in shared memory and executes every root section
-                            in call order; workers run the lock walks below     */
 };
 /* Default execution (no flag):
  *  - bgpq_insert: a level pipeline — one CTA per heap depth applies that depth's
@@ -108,7 +105,9 @@ int bgpq_deletemin_host(bgpq_t* q, uint32_t* out_keys_host, uint32_t* out_vals_h
  * on the persistent CTAs (op j: op_types[j] 0 = INSERT, 1 = DELETEMIN; op_sizes[j] in 1..K).
  * INSERT j reads op_sizes[j] keys at in_keys[in_off[j]]; DELETEMIN j writes at
  * out_keys[j*K] and its entry count to op_count[j].  lin_ticket[j] (nullable) receives
- * the global linearization ticket taken under the root lock.  All device. */
+ * the global linearization ticket taken under the root lock.  All device.
+ * An op size outside 1..K skips the op (op_count = 0 for a DELETEMIN) and sets the sticky
+ * BGPQ_EINVAL reported by the next bgpq_size(). */
 int bgpq_run_mixed(bgpq_t* q, const uint8_t* op_types, const uint32_t* op_sizes,
                    const uint64_t* in_off, uint64_t n_ops, const uint32_t* in_keys,
                    const uint32_t* in_vals, uint32_t* out_keys, uint32_t* out_vals,
@@ -131,6 +130,35 @@ int bgpq_grid(bgpq_t* q);
 
 /* Number of kernels this library has launched in the process (for bench gpu_launches). */
 uint64_t bgpq_launch_count(void);
+
+/* Test / profiling extensions (not part of the minimal ABI).
+ * bgpq_set_debug: process-wide switches read at each call (0 = product behaviour):
+ *   8   accumulate thread-0 cycle timers in the header (read with bgpq_timers);
+ *   16  run deletemin-only calls on the per-node-lock engine instead of the top CTA;
+ *   64  register-window merge path instead of the warp-cooperative one on the top CTA;
+ *   128 light top-CTA timers (plan / phase A / phase B).
+ * bgpq_timers: copies the 32 uint64 cycle counters of the handle to out32 (host);
+ * synchronizes the device. */
+int bgpq_set_debug(uint32_t bits);
+int bgpq_timers(bgpq_t* q, uint64_t* out32);
+
+/* Test extension: run one device primitive of the hot path on n_cases independent cases
+ * (one CTA each; all pointers DEVICE, stream-ordered, no synchronization).  Case c reads
+ * Z = zk[c*K .. c*K+na[c]), W = wk[c*K .. c*K+nb[c]) (sorted, values zv / wv when values != 0)
+ * and writes X to xk[c*2K ..] and Y to yk[c*2K ..]:
+ *   variant 0: SORT_SPLIT as the lock / pipeline executions run it (bitonic split for
+ *              full keys-only batches at K >= 512, register-window merge path otherwise):
+ *              X = the ma smallest of Z u W, Y = the rest, both ascending;
+ *   variant 1: the same split as the top CTA's 256-thread groups run it (warp-cooperative
+ *              merge path; bitonic for full keys-only batches at K >= 512);
+ *   variant 2: the top CTA's register-window merge path (bgpq_set_debug bit 64);
+ *   variant 3: Sort(items) (Alg.1 l.2): X = the na entries of Z sorted (W, nb, ma unused).
+ * Requires 0 <= na, nb <= K, ma <= na + nb (full batches na = nb = ma = K for the bitonic
+ * path).  Equal keys may carry their values in any order (reading R9). */
+int bgpq_test_prim(int variant, uint32_t K, int values, const uint32_t* zk, const uint32_t* zv,
+                   const uint32_t* wk, const uint32_t* wv, const uint32_t* na, const uint32_t* nb,
+                   const uint32_t* ma, uint32_t n_cases, uint32_t* xk, uint32_t* xv, uint32_t* yk,
+                   uint32_t* yv, void* stream);
 
 int bgpq_last_error(void);
 const char* bgpq_last_error_msg(void); /* CUDA error string of the last BGPQ_ECUDA */

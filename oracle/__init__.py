@@ -196,14 +196,15 @@ def check_invariants(K, cap, heap_size, root_size, pb_size, node_keys, states):
     return int(rc), int(where.value)
 
 
-def replay(ops, K=None):
+def replay(ops, q=None):
     """Replay a linearization log through OraclePQ.
 
     ``ops`` is an iterable of (kind, payload) in linearization (ticket) order:
-    kind 0 = insert, payload = (keys, vals); kind 1 = deletemin, payload = size.
+    kind 0 = insert, payload = (keys, vals or None); kind 1 = deletemin, payload = size.
     Returns the list of (keys, vals) the oracle gives each deletemin (P:390-394:
-    x_{k+1} = min_r(I_k - D_k), or all of I_k - D_k if fewer than r remain)."""
-    q = OraclePQ()
+    x_{k+1} = min_r(I_k - D_k), or all of I_k - D_k if fewer than r remain).  ``q``: an
+    OraclePQ to replay into (its state after the log is then available to the caller)."""
+    q = OraclePQ() if q is None else q
     res = []
     for kind, payload in ops:
         if kind == 0:

@@ -19,11 +19,14 @@ _CSRC = os.path.join(_HERE, "csrc")
 _INCLUDE = os.path.join(os.path.dirname(_HERE), "include")
 LIB_PATH = os.environ.get("BGPQ_LIB") or os.path.join(_HERE, "libbgpq.so")
 
-NVCC_FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
-              "-Xptxas", "-v", "-shared", "-Xcompiler", "-fPIC"]
+NVCC_ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
+NVCC_FLAGS = [*NVCC_ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC"]
+BUILD_DIR = os.path.join(_HERE, "build")
+# one object per (K, values) kernel table + the host-side C ABI (compiled in parallel)
+KERNEL_UNITS = [(k, v) for k in (64, 128, 256, 512, 1024) for v in (0, 1)]
 
 BGPQ_OK, BGPQ_EINVAL, BGPQ_ENOMEM, BGPQ_EFULL, BGPQ_ECUDA = 0, -1, -2, -3, -4
-FLAG_VALUES, FLAG_SERIAL, FLAG_LOCKS, FLAG_SERVER = 1, 2, 4, 8
+FLAG_VALUES, FLAG_SERIAL, FLAG_LOCKS = 1, 2, 4
 # GPU node-state encoding (bgpq_ops.cuh); the oracle's encoding differs (see to_oracle_states)
 ST_EMPTY, ST_AVAIL, ST_TARGET, ST_MARKED = 0, 1, 2, 3
 STAT_NAMES = ("ins_ops", "ins_heapify_ops", "ins_levels", "ins_noop", "ins_swap", "ins_merge",
@@ -36,17 +39,39 @@ def _sources():
     return [os.path.join(_CSRC, f) for f in sorted(os.listdir(_CSRC))] + [os.path.join(_INCLUDE, "bgpq.h")]
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    """Compile libbgpq.so for sm_100a in-tree (nvcc cross-compiles without a GPU)."""
+def build(force: bool = False, verbose: bool = False, jobs: int | None = None) -> str:
+    """Compile libbgpq.so for sm_100a in-tree (nvcc cross-compiles without a GPU): the kernel
+    tables of every (K, values) instantiation and the C ABI as separate objects, compiled in
+    parallel, linked with nvcc -shared."""
     newest = max(os.path.getmtime(p) for p in _sources())
-    if force or not os.path.exists(LIB_PATH) or os.path.getmtime(LIB_PATH) < newest:
-        cmd = ["nvcc", *NVCC_FLAGS, "-o", LIB_PATH + ".tmp", os.path.join(_CSRC, "bgpq_api.cu")]
-        r = subprocess.run(cmd, capture_output=True, text=True)
-        if r.returncode != 0:
-            raise RuntimeError("nvcc failed:\n" + r.stderr[-4000:])
-        if verbose:
-            print(r.stderr)
-        os.replace(LIB_PATH + ".tmp", LIB_PATH)
+    if not (force or not os.path.exists(LIB_PATH) or os.path.getmtime(LIB_PATH) < newest):
+        return LIB_PATH
+    os.makedirs(BUILD_DIR, exist_ok=True)
+    units = [([f"-DBGPQ_K={k}", f"-DBGPQ_V={v}"], os.path.join(_CSRC, "bgpq_kernels.cu"),
+              os.path.join(BUILD_DIR, f"kern_{k}_{v}.o")) for k, v in KERNEL_UNITS]
+    units.append(([], os.path.join(_CSRC, "bgpq_api.cu"), os.path.join(BUILD_DIR, "api.o")))
+    units.append(([], os.path.join(_CSRC, "bgpq_testprim.cu"), os.path.join(BUILD_DIR, "testprim.o")))
+    jobs = jobs or max(1, min(len(units), os.cpu_count() or 1))
+    pending, running, logs = list(units), [], []
+    while pending or running:
+        while pending and len(running) < jobs:
+            defs, src, obj = pending.pop(0)
+            cmd = ["nvcc", *NVCC_FLAGS, *(["-Xptxas", "-v"] if verbose else []), *defs, "-c", src, "-o", obj]
+            running.append((subprocess.Popen(cmd, stdout=subprocess.PIPE, stderr=subprocess.STDOUT, text=True), obj))
+        p, obj = running.pop(0)
+        out, _ = p.communicate()
+        logs.append(out)
+        if p.returncode != 0:
+            for q, _ in running:
+                q.kill()
+            raise RuntimeError(f"nvcc failed for {obj}:\n" + out[-4000:])
+    cmd = ["nvcc", *NVCC_ARCH, "-shared", "-o", LIB_PATH + ".tmp", *(u[2] for u in units)]
+    r = subprocess.run(cmd, capture_output=True, text=True)
+    if r.returncode != 0:
+        raise RuntimeError("nvcc link failed:\n" + r.stderr[-4000:])
+    if verbose:
+        print("".join(logs))
+    os.replace(LIB_PATH + ".tmp", LIB_PATH)
     return LIB_PATH
 
 
@@ -79,6 +104,10 @@ def lib():
         L.bgpq_set_grid.argtypes = [_vp, ctypes.c_int]
         L.bgpq_grid.argtypes = [_vp]
         L.bgpq_launch_count.restype = _u64
+        L.bgpq_set_debug.argtypes = [ctypes.c_uint32]
+        L.bgpq_timers.argtypes = [_vp, _vp]
+        L.bgpq_test_prim.argtypes = [ctypes.c_int, ctypes.c_uint32, ctypes.c_int] + [_vp] * 7 + \
+            [ctypes.c_uint32] + [_vp] * 5
         L.bgpq_strerror.restype = ctypes.c_char_p
         L.bgpq_last_error_msg.restype = ctypes.c_char_p
         _lib = L
@@ -89,7 +118,8 @@ def lib():
 EXPORTS = ("bgpq_create", "bgpq_create_ex", "bgpq_destroy", "bgpq_insert", "bgpq_deletemin",
            "bgpq_size", "bgpq_insert_host", "bgpq_deletemin_host", "bgpq_run_mixed", "bgpq_dump",
            "bgpq_slots", "bgpq_stats", "bgpq_set_grid", "bgpq_grid", "bgpq_launch_count",
-           "bgpq_last_error", "bgpq_last_error_msg", "bgpq_strerror")
+           "bgpq_last_error", "bgpq_last_error_msg", "bgpq_strerror", "bgpq_set_debug", "bgpq_timers",
+           "bgpq_test_prim")
 
 
 class BGPQError(RuntimeError):
@@ -106,6 +136,35 @@ def _ptr(t):
     if t is None:
         return None
     return ctypes.c_void_p(t.data_ptr())
+
+
+_U32_DTYPES = None
+
+
+def _dev_buf(t, n, name, dtypes=None):
+    """Validate a caller tensor before its raw pointer crosses the C ABI: CUDA, contiguous,
+    a 4-byte integer dtype (uint32 bit patterns), at least n entries."""
+    global _U32_DTYPES
+    if t is None:
+        return None
+    import torch
+    if _U32_DTYPES is None:
+        _U32_DTYPES = tuple(d for d in (torch.int32, getattr(torch, "uint32", None)) if d is not None)
+    ok_dtypes = dtypes or _U32_DTYPES
+    if not t.is_cuda:
+        raise ValueError(f"{name}: must be a CUDA tensor")
+    if t.dtype not in ok_dtypes:
+        raise ValueError(f"{name}: dtype {t.dtype} not in {ok_dtypes}")
+    if not t.is_contiguous():
+        raise ValueError(f"{name}: must be contiguous")
+    if t.numel() < n:
+        raise ValueError(f"{name}: {t.numel()} entries < {n} required")
+    return ctypes.c_void_p(t.data_ptr())
+
+
+def set_debug(bits: int):
+    """Process-wide test switches of the library (include/bgpq.h bgpq_set_debug)."""
+    _check(lib().bgpq_set_debug(int(bits)))
 
 
 def _stream(stream):
@@ -126,20 +185,20 @@ class BGPQ:
     torch stream, exactly like the C calls they forward to."""
 
     def __init__(self, capacity: int, K: int = 1024, values: bool = True, serial: bool = False,
-                 locks: bool = False, server: bool = False):
+                 locks: bool = False):
         """serial: one CTA, one operation at a time (layout equals the sequential model);
         default: insert calls as a level pipeline, deletemin calls on a top CTA with walker
         CTAs, mixed calls with per-node locks; locks=True: per-node-lock execution for every
-        call; server: root-server execution."""
+        call."""
         if K not in VALID_K:
             raise ValueError(f"K must be one of {VALID_K}")
         flags = ((FLAG_VALUES if values else 0) | (FLAG_SERIAL if serial else 0)
-                 | (FLAG_LOCKS if locks else 0) | (FLAG_SERVER if server else 0))
+                 | (FLAG_LOCKS if locks else 0))
         self._h = lib().bgpq_create_ex(int(capacity), int(K), flags)
         if not self._h:
             raise BGPQError(f"bgpq_create failed ({lib().bgpq_last_error()})")
         self.K, self.capacity, self.values, self.serial = int(K), int(capacity), values, serial
-        self.locks = not server
+        self.locks = locks
 
     def close(self):
         if getattr(self, "_h", None):
@@ -154,7 +213,9 @@ class BGPQ:
     # -- hot path -------------------------------------------------------------------------
     def insert(self, keys, vals=None, stream=None):
         """BGPQ_INSERT of keys (device tensor, n entries) in ceil(n/K) batches."""
-        _check(lib().bgpq_insert(self._h, _ptr(keys), _ptr(vals), keys.numel(), _stream(stream)))
+        n = keys.numel()
+        _check(lib().bgpq_insert(self._h, _dev_buf(keys, n, "keys"), _dev_buf(vals, n, "vals"), n,
+                                 _stream(stream)))
 
     def deletemin(self, n, out_keys=None, out_vals=None, d_count=None, stream=None):
         """BGPQ_DELETEMIN of n keys; returns (out_keys, out_vals) device tensors (length n;
@@ -164,8 +225,9 @@ class BGPQ:
             out_keys = torch.empty(n, dtype=torch.int32, device="cuda")
         if out_vals is None and self.values:
             out_vals = torch.empty(n, dtype=torch.int32, device="cuda")
-        _check(lib().bgpq_deletemin(self._h, _ptr(out_keys), _ptr(out_vals), int(n), _ptr(d_count),
-                                    _stream(stream)))
+        import torch
+        _check(lib().bgpq_deletemin(self._h, _dev_buf(out_keys, n, "out_keys"), _dev_buf(out_vals, n, "out_vals"),
+                                    int(n), _dev_buf(d_count, 1, "d_count", (torch.int64,)), _stream(stream)))
         return out_keys, out_vals
 
     def size(self, stream=None) -> int:
@@ -175,11 +237,19 @@ class BGPQ:
 
     # -- host-buffer variants (e2e) ---------------------------------------------------------
     def insert_host(self, keys: np.ndarray, vals: np.ndarray | None = None, stream=None):
+        if keys.dtype.itemsize != 4 or not keys.flags.c_contiguous:
+            raise ValueError("keys: contiguous 4-byte integers required")
+        if vals is not None and (vals.dtype.itemsize != 4 or len(vals) < len(keys) or not vals.flags.c_contiguous):
+            raise ValueError("vals: contiguous 4-byte integers, len >= len(keys) required")
         _check(lib().bgpq_insert_host(self._h, keys.ctypes.data_as(_vp),
                                       None if vals is None else vals.ctypes.data_as(_vp),
                                       len(keys), _stream(stream)))
 
     def deletemin_host(self, n, out_keys: np.ndarray, out_vals: np.ndarray | None = None, stream=None):
+        if out_keys.dtype.itemsize != 4 or len(out_keys) < n or not out_keys.flags.c_contiguous:
+            raise ValueError("out_keys: contiguous 4-byte integers, len >= n required")
+        if out_vals is not None and (out_vals.dtype.itemsize != 4 or len(out_vals) < n):
+            raise ValueError("out_vals: 4-byte integers, len >= n required")
         cnt = _u64(0)
         _check(lib().bgpq_deletemin_host(self._h, out_keys.ctypes.data_as(_vp),
                                          None if out_vals is None else out_vals.ctypes.data_as(_vp),
@@ -215,23 +285,34 @@ class BGPQ:
         _check(lib().bgpq_stats(self._h, out.ctypes.data_as(_vp), len(STAT_NAMES)))
         return dict(zip(STAT_NAMES, (int(x) for x in out)))
 
-    TIMER_NAMES = {0: "srv_total", 1: "srv_batch_wait", 2: "srv_tar_wait", 3: "srv_home_wait",
-                   4: "srv_task_wait", 5: "srv_merge", 6: "srv_ins", 7: "srv_del", 8: "srv_merges_n",
-                   16: "w_sort", 17: "w_ins", 18: "w_del", 19: "w_idle", 20: "w_ins_n", 21: "w_del_n",
-                   22: "w_sort_n", 9: "d_start", 10: "d_emit", 11: "d_refill", 12: "d_pb",
-                   13: "d_decide", 14: "d_lr", 15: "d_cy", 24: "d_extract", 25: "d_exit", 26: "d_lend"}
-
-    def timers(self) -> dict:
-        """Cycle counters of the server-mode kernel (cumulative; debug aid)."""
+    def timers(self) -> np.ndarray:
+        """The 32 cumulative cycle counters of the handle (set_debug(8 | 128); debug aid)."""
         out = np.zeros(32, np.uint64)
         _check(lib().bgpq_timers(self._h, out.ctypes.data_as(_vp)))
-        return {nm: int(out[i]) for i, nm in self.TIMER_NAMES.items()}
+        return out
 
     def set_grid(self, ctas: int):
         _check(lib().bgpq_set_grid(self._h, int(ctas)))
 
     def grid(self) -> int:
         return int(lib().bgpq_grid(self._h))
+
+
+def test_prim(variant: int, K: int, zk, wk, na, nb, ma, zv=None, wv=None):
+    """Run one hot-path device primitive on a batch of cases (include/bgpq.h bgpq_test_prim).
+    zk / wk: [n_cases, K] int32 CUDA tensors; na / nb / ma: [n_cases] int32 CUDA tensors.
+    Returns (xk, xv, yk, yv) as [n_cases, 2K] CUDA tensors (xv / yv None without values)."""
+    import torch
+    n = zk.shape[0]
+    values = zv is not None
+    xk = torch.zeros((n, 2 * K), dtype=torch.int32, device=zk.device)
+    yk = torch.zeros_like(xk)
+    xv = torch.zeros_like(xk) if values else None
+    yv = torch.zeros_like(xk) if values else None
+    _check(lib().bgpq_test_prim(int(variant), int(K), int(values), _ptr(zk), _ptr(zv), _ptr(wk), _ptr(wv),
+                                _ptr(na), _ptr(nb), _ptr(ma), int(n), _ptr(xk), _ptr(xv), _ptr(yk), _ptr(yv),
+                                _stream(None)))
+    return xk, xv, yk, yv
 
 
 def to_oracle_states(gpu_states: np.ndarray) -> np.ndarray:

@@ -11,23 +11,18 @@
 #include <cstring>
 
 #include "../../include/bgpq.h"
-#include "bgpq_locks.cuh"
-#include "bgpq_pipe.cuh"
-#include "bgpq_server.cuh"
-#include "bgpq_dtop.cuh"
-#include "bgpq_pipe2.cuh"
+#include "bgpq_ktab.h"
 
 using namespace bgpqd;
 
 namespace {
 
-constexpr int NT = 512;  // threads per CTA (the paper's block size)
+
 
 thread_local int g_last_error = BGPQ_OK;
 thread_local char g_last_msg[256] = "";
 std::atomic<unsigned long long> g_launches{0};
-unsigned g_debug = 0;  // test-only switches, from env BGPQ_DEBUG
-volatile u32* g_prog = nullptr;  // test-only progress log (host-mapped), bgpq_debug_progress()
+unsigned g_debug = 0;  // test-only switches (bgpq_set_debug)
 
 int fail(int code) {
   g_last_error = code;
@@ -54,236 +49,37 @@ struct bgpq {
   int sm_count = 0;
   int occ = 0;         // co-resident CTAs per SM for this K
   int grid_req = 0;    // 0 auto, else exact
-  SrvArgs srv{};           // server-mode rings and control words (device)
   PipeArgs pipe{};         // insert-pipeline rings (allocated at the first pipelined insert)
   bool pipe_ok = false;
   int pipe_grid = 0;
-  bool srv_ok = false;
-  int srv_grid = 0;
   DtArgs dt{};             // deletemin top-CTA execution: walker task list (bgpq_dtop.cuh)
   bool dt_ok = false;
   u32* stage_k = nullptr;  // staging for the *_host calls
   u32* stage_v = nullptr;
   u64* stage_cnt = nullptr;
   u64 stage_n = 0;
+  bool attr_dt = false;    // kernel attributes set / occupancy checked on q->device
+  bool attr_pipe = false;
 };
 
 namespace {
 
-template <int K, bool V>
-struct KernelInfo {
-  // the per-node-lock execution (bgpq_locks.cuh): NT compute threads + one lock warp
-  static int occupancy(int* out_occ) {
-    auto kern = bgpq_locks_kernel<K, V, NT>;
-    const size_t smem = locks_smem_bytes<K, V>();
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (e != cudaSuccess) return -1;
-    int occ = 0;
-    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, NT + 32, smem);
-    if (e != cudaSuccess) return -1;
-    *out_occ = occ;
-    return 0;
-  }
-  static cudaError_t launch(int grid, const HeapArgs& H, const CallArgs& C, cudaStream_t s) {
-    bgpq_locks_kernel<K, V, NT><<<grid, NT + 32, locks_smem_bytes<K, V>(), s>>>(H, C);
-    g_launches.fetch_add(1);
-    return cudaGetLastError();
-  }
-  static int srv_occupancy(int* out_occ) {
-    auto kern = bgpq_srv_kernel<K, V, NT>;
-    const size_t smem = SrvShape<K, V, NT>::smem;
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (e != cudaSuccess) return -1;
-    int occ = 0;
-    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, NT + 32, smem);
-    if (e != cudaSuccess) return -1;
-    *out_occ = occ;
-    return 0;
-  }
-  static cudaError_t srv_launch(int grid, const HeapArgs& H, const CallArgs& C, const SrvArgs& A,
-                                cudaStream_t s) {
-    bgpq_srv_kernel<K, V, NT><<<grid, NT + 32, SrvShape<K, V, NT>::smem, s>>>(H, C, A);
-    g_launches.fetch_add(1);
-    return cudaGetLastError();
-  }
-  static cudaError_t dt_launch(int grid, const HeapArgs& H, const CallArgs& C, const DtArgs& D, cudaStream_t s) {
-    static bool attr = false;
-    auto kern = bgpq_dtop_kernel<K, V>;
-    const size_t smem = dt_smem_bytes<K, V>();
-    if (!attr) {
-      cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-      if (e != cudaSuccess) return e;
-      int occ = 0;
-      e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, DT_BLOCK, smem);
-      if (e != cudaSuccess) return e;
-      if (occ < 1) return cudaErrorLaunchOutOfResources;
-      attr = true;
-    }
-    kern<<<grid, DT_BLOCK, smem, s>>>(H, C, D);
-    g_launches.fetch_add(1);
-    return cudaGetLastError();
-  }
-  static int srv_top_nodes() { return SrvShape<K, V, NT>::NTOP; }
-  static int pipe_occupancy(int* out_occ) {
-    auto kern = bgpq_ins_pipe_kernel<K, V, NT>;
-    const size_t smem = pipe_smem_bytes<K, V>();
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (e != cudaSuccess) return -1;
-    int occ = 0;
-    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, NT, smem);
-    if (e != cudaSuccess) return -1;
-    *out_occ = occ;
-    return 0;
-  }
-  static cudaError_t pipe_launch(int grid, const HeapArgs& H, const PipeArgs& P, const CallArgs& C,
-                                 cudaStream_t s) {
-    if (g_debug & 32u) {  // test switch: the synchronous pipeline (bgpq_pipe.cuh)
-      bgpq_ins_pipe_kernel<K, V, NT><<<grid, NT, pipe_smem_bytes<K, V>(), s>>>(H, P, C);
-    } else {
-      static bool attr = false;
-      auto kern = bgpq_ins_pipe2_kernel<K, V, NT>;
-      const size_t smem = pipe2_smem_bytes<K, V>();
-      if (!attr) {
-        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        if (e != cudaSuccess) return e;
-        attr = true;
-      }
-      kern<<<grid, NT + 64, smem, s>>>(H, P, C);
-    }
-    g_launches.fetch_add(1);
-    return cudaGetLastError();
-  }
-};
-
-int occupancy_for(u32 K, bool V, int* occ) {
-#define BGPQ_CASE(KK)                                                                \
-  case KK:                                                                           \
-    return V ? KernelInfo<KK, true>::occupancy(occ) : KernelInfo<KK, false>::occupancy(occ);
+// ---- per-K kernel tables (bgpq_kernels.cu, one translation unit per K) ------------------
+const KTable* ktab(u32 K, bool V) {
   switch (K) {
-    BGPQ_CASE(64)
-    BGPQ_CASE(128)
-    BGPQ_CASE(256)
-    BGPQ_CASE(512)
-    BGPQ_CASE(1024)
-    default:
-      return -1;
+    case 64: return V ? &ktab_64_v() : &ktab_64_k();
+    case 128: return V ? &ktab_128_v() : &ktab_128_k();
+    case 256: return V ? &ktab_256_v() : &ktab_256_k();
+    case 512: return V ? &ktab_512_v() : &ktab_512_k();
+    case 1024: return V ? &ktab_1024_v() : &ktab_1024_k();
+    default: return nullptr;
   }
-#undef BGPQ_CASE
 }
+const KTable* ktab(const bgpq* q) { return ktab(q->K, (q->flags & BGPQ_FLAG_VALUES) != 0); }
 
-cudaError_t launch_for(u32 K, bool V, int grid, const HeapArgs& H, const CallArgs& C, cudaStream_t s) {
-#define BGPQ_CASE(KK)                                                                        \
-  case KK:                                                                                   \
-    return V ? KernelInfo<KK, true>::launch(grid, H, C, s) : KernelInfo<KK, false>::launch(grid, H, C, s);
-  switch (K) {
-    BGPQ_CASE(64)
-    BGPQ_CASE(128)
-    BGPQ_CASE(256)
-    BGPQ_CASE(512)
-    BGPQ_CASE(1024)
-    default:
-      return cudaErrorInvalidValue;
-  }
-#undef BGPQ_CASE
-}
-
-int srv_occupancy_for(u32 K, bool V, int* occ) {
-#define BGPQ_CASE(KK)                                                                        \
-  case KK:                                                                                   \
-    return V ? KernelInfo<KK, true>::srv_occupancy(occ) : KernelInfo<KK, false>::srv_occupancy(occ);
-  switch (K) {
-    BGPQ_CASE(64)
-    BGPQ_CASE(128)
-    BGPQ_CASE(256)
-    BGPQ_CASE(512)
-    BGPQ_CASE(1024)
-    default:
-      return -1;
-  }
-#undef BGPQ_CASE
-}
-
-int srv_top_for(u32 K, bool V) {
-#define BGPQ_CASE(KK)                                                                        \
-  case KK:                                                                                   \
-    return V ? KernelInfo<KK, true>::srv_top_nodes() : KernelInfo<KK, false>::srv_top_nodes();
-  switch (K) {
-    BGPQ_CASE(64)
-    BGPQ_CASE(128)
-    BGPQ_CASE(256)
-    BGPQ_CASE(512)
-    BGPQ_CASE(1024)
-    default:
-      return 0;
-  }
-#undef BGPQ_CASE
-}
-
-cudaError_t srv_launch_for(u32 K, bool V, int grid, const HeapArgs& H, const CallArgs& C, const SrvArgs& A,
-                           cudaStream_t s) {
-#define BGPQ_CASE(KK)                                                                        \
-  case KK:                                                                                   \
-    return V ? KernelInfo<KK, true>::srv_launch(grid, H, C, A, s) : KernelInfo<KK, false>::srv_launch(grid, H, C, A, s);
-  switch (K) {
-    BGPQ_CASE(64)
-    BGPQ_CASE(128)
-    BGPQ_CASE(256)
-    BGPQ_CASE(512)
-    BGPQ_CASE(1024)
-    default:
-      return cudaErrorInvalidValue;
-  }
-#undef BGPQ_CASE
-}
-
-cudaError_t dt_launch_for(u32 K, bool V, int grid, const HeapArgs& H, const CallArgs& C, const DtArgs& D,
-                          cudaStream_t s) {
-#define BGPQ_CASE(KK)                                                                        \
-  case KK:                                                                                   \
-    return V ? KernelInfo<KK, true>::dt_launch(grid, H, C, D, s) : KernelInfo<KK, false>::dt_launch(grid, H, C, D, s);
-  switch (K) {
-    BGPQ_CASE(64)
-    BGPQ_CASE(128)
-    BGPQ_CASE(256)
-    BGPQ_CASE(512)
-    BGPQ_CASE(1024)
-    default:
-      return cudaErrorInvalidValue;
-  }
-#undef BGPQ_CASE
-}
-
-int pipe_occupancy_for(u32 K, bool V, int* occ) {
-#define BGPQ_CASE(KK)                                                                        \
-  case KK:                                                                                   \
-    return V ? KernelInfo<KK, true>::pipe_occupancy(occ) : KernelInfo<KK, false>::pipe_occupancy(occ);
-  switch (K) {
-    BGPQ_CASE(64)
-    BGPQ_CASE(128)
-    BGPQ_CASE(256)
-    BGPQ_CASE(512)
-    BGPQ_CASE(1024)
-    default:
-      return -1;
-  }
-#undef BGPQ_CASE
-}
-
-cudaError_t pipe_launch_for(u32 K, bool V, int grid, const HeapArgs& H, const PipeArgs& P, const CallArgs& C,
-                            cudaStream_t s) {
-#define BGPQ_CASE(KK)                                                                        \
-  case KK:                                                                                   \
-    return V ? KernelInfo<KK, true>::pipe_launch(grid, H, P, C, s) : KernelInfo<KK, false>::pipe_launch(grid, H, P, C, s);
-  switch (K) {
-    BGPQ_CASE(64)
-    BGPQ_CASE(128)
-    BGPQ_CASE(256)
-    BGPQ_CASE(512)
-    BGPQ_CASE(1024)
-    default:
-      return cudaErrorInvalidValue;
-  }
-#undef BGPQ_CASE
+cudaError_t counted(cudaError_t e) {
+  if (e == cudaSuccess) g_launches.fetch_add(1);
+  return e;
 }
 
 bool valid_K(u32 K) { return K == 64 || K == 128 || K == 256 || K == 512 || K == 1024; }
@@ -311,21 +107,22 @@ u32 depth_host(u32 i) {
   return d;
 }
 
-bool server_mode(const bgpq* q) { return (q->flags & BGPQ_FLAG_SERVER) && !(q->flags & BGPQ_FLAG_SERIAL); }
+// Insert-only calls in the default execution run as a level pipeline (bgpq_pipe2.cuh).
+bool pipe_mode(const bgpq* q) { return !(q->flags & (BGPQ_FLAG_SERIAL | BGPQ_FLAG_LOCKS)); }
 
-// Insert-only calls in the default execution run as a level pipeline (bgpq_pipe.cuh).
-bool pipe_mode(const bgpq* q) {
-  return !(q->flags & (BGPQ_FLAG_SERIAL | BGPQ_FLAG_LOCKS | BGPQ_FLAG_SERVER));
-}
-
-bool ensure_pipe(bgpq* q) {
-  if (q->pipe_ok) return true;
+// Allocates the pipeline rings and checks that its grid (one CTA per SM: root stage, one stage
+// per heap depth, sorters) is co-resident.  Returns BGPQ_OK, BGPQ_ENOMEM (allocation),
+// BGPQ_ECUDA (attribute / occupancy query) or BGPQ_EINVAL (heap deeper than the grid holds
+// stages for; cannot happen for capacities that fit a B200's memory).
+int ensure_pipe(bgpq* q) {
+  if (q->pipe_ok) return BGPQ_OK;
   const bool V = (q->flags & BGPQ_FLAG_VALUES) != 0;
   const u32 depth = depth_host(q->cap_nodes);
   int occ = 0;
-  if (pipe_occupancy_for(q->K, V, &occ) != 0 || occ < 1) return false;
-  const int grid = q->sm_count;  // one CTA per SM, all co-resident
-  if ((int)depth + 2 > grid || depth >= PIPE_MAXL) return false;
+  if (ktab(q)->pipe_prepare(&occ) != cudaSuccess) return fail(BGPQ_ECUDA);
+  if (occ < 1) return fail(BGPQ_ECUDA);
+  const int grid = q->sm_count;  // one CTA per SM, all co-resident (occ >= 1)
+  if ((int)depth + 2 > grid || depth >= PIPE_MAXL) return fail(BGPQ_EINVAL);
   PipeArgs& P = q->pipe;
   const size_t kb = (size_t)q->K * sizeof(u32);
   bool ok = cudaMalloc(&P.ctl, PC_WORDS * sizeof(u32)) == cudaSuccess;
@@ -338,70 +135,74 @@ bool ensure_pipe(bgpq* q) {
     ok = ok && cudaMalloc(&P.sbv, PIPE_NSB * kb) == cudaSuccess;
     ok = ok && cudaMalloc(&P.rv, (size_t)PIPE_MAXL * PIPE_NL * kb) == cudaSuccess;
   }
+  if (!ok) {
+    cudaGetLastError();
+    return fail(BGPQ_ENOMEM);
+  }
   P.depth = depth;
   q->pipe_grid = grid;
-  q->pipe_ok = ok;
-  return ok;
+  q->pipe_ok = true;
+  return BGPQ_OK;
 }
 
 // Deletemin-only calls in the default execution: top CTA + walkers (bgpq_dtop.cuh).
-// BGPQ_DEBUG bit 16 routes them to the per-op lock execution instead (A/B comparisons).
+// Debug bit 16 routes them to the per-node-lock execution instead (A/B comparisons).
 bool dt_mode(const bgpq* q) { return pipe_mode(q) && !(g_debug & 16u); }
 
-bool ensure_dt(bgpq* q) {
-  if (q->dt_ok) return true;
+// Walker task list: one entry per hand-off (at most one per refill node, <= cap_nodes) plus
+// one ticket per walker CTA past the final count (each walker takes tickets until it sees
+// the count), so cap_nodes + 2 + grid entries are ever indexed.
+size_t dt_tasks(const bgpq* q) { return (size_t)q->cap_nodes + 2 + (size_t)q->sm_count; }
+
+int ensure_dt(bgpq* q) {
+  if (q->dt_ok) return BGPQ_OK;
+  const bool V = (q->flags & BGPQ_FLAG_VALUES) != 0;
+  int occ = 0;
+  if (ktab(q)->dt_prepare(&occ) != cudaSuccess || occ < 1) return fail(BGPQ_ECUDA);
   DtArgs& D = q->dt;
-  const size_t n = (size_t)q->cap_nodes + 2;
+  const size_t n = dt_tasks(q);
   bool ok = cudaMalloc(&D.task_node, n * sizeof(u32)) == cudaSuccess;
   ok = ok && cudaMalloc(&D.task_seq, n * sizeof(u32)) == cudaSuccess;
   ok = ok && cudaMalloc(&D.ctl, 32 * sizeof(u32)) == cudaSuccess;
-  ok = ok && cudaMemset(D.task_seq, 0, n * sizeof(u32)) == cudaSuccess;
-  ok = ok && cudaMemset(D.ctl, 0, 32 * sizeof(u32)) == cudaSuccess;
+  if (!ok) {
+    cudaGetLastError();
+    return fail(BGPQ_ENOMEM);
+  }
+  if (cudaMemset(D.task_seq, 0, n * sizeof(u32)) != cudaSuccess ||
+      cudaMemset(D.ctl, 0, 32 * sizeof(u32)) != cudaSuccess)
+    return fail(BGPQ_ECUDA);
   D.epoch = 0;
-  q->dt_ok = ok;
-  return ok;
+  q->dt_ok = true;
+  return BGPQ_OK;
 }
 
 int run_call(bgpq* q, const CallArgs& C, cudaStream_t s) {
   const bool V = (q->flags & BGPQ_FLAG_VALUES) != 0;
   if (C.mode == MODE_DELETEMIN && dt_mode(q)) {
-    if (!ensure_dt(q)) return fail(BGPQ_ENOMEM);
+    if (int rc = ensure_dt(q)) return rc;
     DtArgs& D = q->dt;
     D.epoch += 1;
     if (D.epoch == 0) {  // wrapped: clear the stale epochs
       D.epoch = 1;
-      if (cudaMemsetAsync(D.task_seq, 0, ((size_t)q->cap_nodes + 2) * sizeof(u32), s) != cudaSuccess)
-        return fail(BGPQ_ECUDA);
+      if (cudaMemsetAsync(D.task_seq, 0, dt_tasks(q) * sizeof(u32), s) != cudaSuccess) return fail(BGPQ_ECUDA);
     }
     if (cudaMemsetAsync(D.ctl, 0, 2 * sizeof(u32), s) != cudaSuccess) return fail(BGPQ_ECUDA);
-    if (dt_launch_for(q->K, V, q->sm_count, heap_args(q), C, D, s) != cudaSuccess) return fail(BGPQ_ECUDA);
+    if (counted(ktab(q)->dt_launch(q->sm_count, heap_args(q), C, D, s)) != cudaSuccess) return fail(BGPQ_ECUDA);
     return BGPQ_OK;
   }
   if (C.mode == MODE_INSERT && pipe_mode(q)) {
-    if (!ensure_pipe(q)) return fail(BGPQ_ENOMEM);
+    if (int rc = ensure_pipe(q)) return rc;
     const PipeArgs& P = q->pipe;
     bool ok = cudaMemsetAsync(P.ctl, 0, PC_WORDS * sizeof(u32), s) == cudaSuccess;
     ok = ok && cudaMemsetAsync(P.sready, 0, PIPE_NSB * sizeof(u32), s) == cudaSuccess;
     ok = ok && cudaMemsetAsync(P.rflag, 0, (size_t)PIPE_MAXL * PIPE_NL * sizeof(u32), s) == cudaSuccess;
     if (!ok) return fail(BGPQ_ECUDA);
-    if (pipe_launch_for(q->K, V, q->pipe_grid, heap_args(q), P, C, s) != cudaSuccess) return fail(BGPQ_ECUDA);
-    return BGPQ_OK;
-  }
-  if (server_mode(q)) {
-    // reset the per-call control words, publication flags, gate tickets and lend counters
-    const int ntop = srv_top_for(q->K, V);
-    bool ok = cudaMemsetAsync(q->srv.ctl, 0, C_WORDS * sizeof(u32), s) == cudaSuccess;
-    ok = ok && cudaMemsetAsync(q->srv.task_pub, 0, NTASK * sizeof(u32), s) == cudaSuccess;
-    ok = ok && cudaMemsetAsync(q->srv.sready, 0, NSB * sizeof(u32), s) == cudaSuccess;
-    ok = ok && cudaMemsetAsync(q->srv.serving, 0, ntop * sizeof(u32), s) == cudaSuccess;
-    ok = ok && cudaMemsetAsync(q->srv.ret, 0, ntop * sizeof(u32), s) == cudaSuccess;
-    if (!ok) return fail(BGPQ_ECUDA);
-    if (srv_launch_for(q->K, V, q->srv_grid, heap_args(q), C, q->srv, s) != cudaSuccess) return fail(BGPQ_ECUDA);
+    if (counted(ktab(q)->pipe_launch(q->pipe_grid, heap_args(q), P, C, s)) != cudaSuccess) return fail(BGPQ_ECUDA);
     return BGPQ_OK;
   }
   // reset the per-call ticket and fetch counter (header words H_CALL, H_FETCH)
   if (cudaMemsetAsync(q->hdr + H_CALL, 0, 2 * sizeof(u32), s) != cudaSuccess) return fail(BGPQ_ECUDA);
-  if (launch_for(q->K, V, grid_for(q, C.n_ops), heap_args(q), C, s) != cudaSuccess) return fail(BGPQ_ECUDA);
+  if (counted(ktab(q)->locks_launch(grid_for(q, C.n_ops), heap_args(q), C, s)) != cudaSuccess) return fail(BGPQ_ECUDA);
   return BGPQ_OK;
 }
 
@@ -411,8 +212,7 @@ extern "C" {
 
 bgpq_t* bgpq_create_ex(uint64_t capacity, uint32_t K, uint32_t flags) {
   g_last_error = BGPQ_OK;
-  if (const char* d = getenv("BGPQ_DEBUG")) g_debug = (unsigned)atoi(d);
-  if (!valid_K(K) || capacity == 0 || (flags & ~15u)) {
+  if (!valid_K(K) || capacity == 0 || (flags & ~7u)) {
     fail(BGPQ_EINVAL);
     return nullptr;
   }
@@ -435,7 +235,7 @@ bgpq_t* bgpq_create_ex(uint64_t capacity, uint32_t K, uint32_t flags) {
     return nullptr;
   }
   const bool V = (flags & BGPQ_FLAG_VALUES) != 0;
-  if (occupancy_for(K, V, &q->occ) != 0 || q->occ < 1) {
+  if (ktab(K, V)->locks_prepare(&q->occ) != cudaSuccess || q->occ < 1) {
     delete q;
     fail(BGPQ_ECUDA);
     return nullptr;
@@ -447,35 +247,6 @@ bgpq_t* bgpq_create_ex(uint64_t capacity, uint32_t K, uint32_t flags) {
   if (ok) ok = cudaMalloc(&q->hdr, HEADER_WORDS * sizeof(u32)) == cudaSuccess;
   if (ok) ok = cudaMemset(q->meta, 0, q->slots * sizeof(NodeMeta)) == cudaSuccess;
   if (ok) ok = cudaMemset(q->hdr, 0, HEADER_WORDS * sizeof(u32)) == cudaSuccess;
-  if (ok && server_mode(q)) {
-    int socc = 0;
-    if (srv_occupancy_for(K, V, &socc) != 0 || socc < 1) {
-      cudaDeviceSynchronize();
-      bgpq_destroy(q);
-      fail(BGPQ_ECUDA);
-      return nullptr;
-    }
-    q->srv_grid = q->sm_count * socc;  // every CTA co-resident: the server and all workers
-    const int ntop = srv_top_for(K, V);
-    SrvArgs& A = q->srv;
-    memset(&A, 0, sizeof(A));
-    const size_t kb = (size_t)K * sizeof(u32);
-    ok = cudaMalloc(&A.ctl, C_WORDS * sizeof(u32)) == cudaSuccess;
-    ok = ok && cudaMalloc(&A.task, (size_t)NTASK * 8 * sizeof(u32)) == cudaSuccess;
-    ok = ok && cudaMalloc(&A.task_pub, NTASK * sizeof(u32)) == cudaSuccess;
-    ok = ok && cudaMalloc(&A.payk, NTASK * kb) == cudaSuccess;
-    ok = ok && cudaMalloc(&A.sbk, NSB * kb) == cudaSuccess;
-    ok = ok && cudaMalloc(&A.sready, NSB * sizeof(u32)) == cudaSuccess;
-    ok = ok && cudaMalloc(&A.serving, ntop * sizeof(u32)) == cudaSuccess;
-    ok = ok && cudaMalloc(&A.ret, ntop * sizeof(u32)) == cudaSuccess;
-    ok = ok && cudaMalloc(&A.mailk, kb) == cudaSuccess;
-    if (V) {
-      ok = ok && cudaMalloc(&A.payv, NTASK * kb) == cudaSuccess;
-      ok = ok && cudaMalloc(&A.sbv, NSB * kb) == cudaSuccess;
-      ok = ok && cudaMalloc(&A.mailv, kb) == cudaSuccess;
-    }
-    q->srv_ok = ok;
-  }
   if (ok) ok = cudaDeviceSynchronize() == cudaSuccess;
   if (!ok) {
     cudaGetLastError();
@@ -498,9 +269,6 @@ void bgpq_destroy(bgpq_t* q) {
   cudaFree(q->stage_k);
   cudaFree(q->stage_v);
   cudaFree(q->stage_cnt);
-  SrvArgs& A = q->srv;
-  u32* bufs[] = {A.ctl, A.task, A.task_pub, A.payk, A.payv, A.sbk, A.sbv, A.sready, A.serving, A.ret, A.mailk, A.mailv};
-  for (u32* b : bufs) cudaFree(b);
   cudaFree(q->dt.task_node);
   cudaFree(q->dt.task_seq);
   cudaFree(q->dt.ctl);
@@ -522,7 +290,7 @@ int bgpq_insert(bgpq_t* q, const uint32_t* keys, const uint32_t* vals, uint64_t 
   C.in_k = keys;
   C.in_v = (q->flags & BGPQ_FLAG_VALUES) ? vals : nullptr;
   C.debug = g_debug;
-  C.prog = g_prog;
+  C.prog = nullptr;
   return run_call(q, C, (cudaStream_t)stream);
 }
 
@@ -540,7 +308,7 @@ int bgpq_deletemin(bgpq_t* q, uint32_t* out_keys, uint32_t* out_vals, uint64_t n
   C.out_v = (q->flags & BGPQ_FLAG_VALUES) ? out_vals : nullptr;
   C.d_count = reinterpret_cast<ull*>(d_count);
   C.debug = g_debug;
-  C.prog = g_prog;
+  C.prog = nullptr;
   return run_call(q, C, (cudaStream_t)stream);
 }
 
@@ -564,7 +332,7 @@ int bgpq_run_mixed(bgpq_t* q, const uint8_t* op_types, const uint32_t* op_sizes,
   C.op_count = op_count;
   C.lin_ticket = reinterpret_cast<ull*>(lin_ticket);
   C.debug = g_debug;
-  C.prog = g_prog;
+  C.prog = nullptr;
   return run_call(q, C, (cudaStream_t)stream);
 }
 
@@ -664,31 +432,10 @@ int bgpq_stats(bgpq_t* q, uint64_t* out, int n) {
   return BGPQ_OK;
 }
 
-// test-only: allocate (once) and return a 64-word host-mapped progress log
-uint32_t* bgpq_debug_progress(void) {
-  if (!g_prog) {
-    void* h = nullptr;
-    if (cudaHostAlloc(&h, 1024 * sizeof(u32), cudaHostAllocMapped) != cudaSuccess) return nullptr;
-    memset(h, 0, 1024 * sizeof(u32));
-    void* d = nullptr;
-    cudaHostGetDevicePointer(&d, h, 0);
-    g_prog = reinterpret_cast<volatile u32*>(d);
-    return reinterpret_cast<uint32_t*>(h);
-  }
-  return nullptr;
-}
-
 int bgpq_timers(bgpq_t* q, uint64_t* out32) {
   if (!q || !out32) return fail(BGPQ_EINVAL);
   if (cudaDeviceSynchronize() != cudaSuccess) return fail(BGPQ_ECUDA);
   if (cudaMemcpy(out32, q->hdr + H_TIME, 32 * sizeof(u64), cudaMemcpyDeviceToHost) != cudaSuccess) return fail(BGPQ_ECUDA);
-  return BGPQ_OK;
-}
-
-int bgpq_debug_record(bgpq_t* q, uint32_t* out4) {
-  if (!q || !out4) return fail(BGPQ_EINVAL);
-  if (cudaDeviceSynchronize() != cudaSuccess) return fail(BGPQ_ECUDA);
-  if (cudaMemcpy(out4, q->hdr + 60, 16, cudaMemcpyDeviceToHost) != cudaSuccess) return fail(BGPQ_ECUDA);
   return BGPQ_OK;
 }
 
@@ -699,7 +446,12 @@ int bgpq_set_grid(bgpq_t* q, int ctas) {
   return BGPQ_OK;
 }
 
-int bgpq_grid(bgpq_t* q) { return q ? (server_mode(q) ? q->srv_grid : grid_for(q, ~0ull)) : 0; }
+int bgpq_grid(bgpq_t* q) { return q ? grid_for(q, ~0ull) : 0; }
+
+int bgpq_set_debug(uint32_t bits) {
+  g_debug = bits;
+  return BGPQ_OK;
+}
 
 uint64_t bgpq_launch_count(void) { return g_launches.load(); }
 

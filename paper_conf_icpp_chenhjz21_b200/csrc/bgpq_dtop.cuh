@@ -1246,212 +1246,6 @@ __device__ __forceinline__ void dt_top(DTop<K, V>& T) {
   }
 }
 
-// named barriers (aligned forms: the whole warp must execute them convergently, hence the
-// __syncwarp after any lane-0-only code)
-__device__ __forceinline__ void nbar_sync(int id, int n) {
-  __syncwarp();
-  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory");
-}
-__device__ __forceinline__ void nbar_arrive(int id, int n) {
-  __syncwarp();
-  asm volatile("bar.arrive %0, %1;" ::"r"(id), "r"(n) : "memory");
-}
-
-// =========================================================================================
-// Control-warp driver (test switch BGPQ_DEBUG bit 512; measured no faster than dt_top, whose
-// thread-0 decision chain it moves to a dedicated warp).  The decisions of a slot (dt_fast / dt_slow, then dt_plan)
-// run on a dedicated warp: the three groups are released (barrier READY) as soon as the plan
-// of the next slot is written, and the control warp then issues the slot's helper requests and
-// the output copy while the groups merge; the groups report phase A done on barrier DONE.
-// =========================================================================================
-template <int K, bool V>
-__device__ __forceinline__ void dt_groups2(DTop<K, V>& T) {
-  DtCtl* c = T.c;
-  const int tid = threadIdx.x, g = tid / DT_GT, gt = tid % DT_GT;
-  const bool mwin = (T.C.debug & 64u) != 0;
-  constexpr int NB_ = DT_NTC + 32;
-  mbar_wait(&c->lbar, 0);
-  for (;;) {
-    nbar_sync(DT_BAR_READY, NB_);
-    const u32 pf = c->p_flags;
-    if (pf == DT_NONE) break;
-    if (pf & F_JOBS) {
-      T.run_jobs();
-      nbar_arrive(DT_BAR_DONE, NB_);
-      continue;
-    }
-    const u32 w_sbi = c->p_sbi, w_spar = c->p_spar, w_rwait = c->p_rwait, w_rbi = c->p_rbi, w_rpar = c->p_rpar;
-    const bool lt = (T.C.debug & 128u) != 0;
-    const ull ta = (lt && gt == 0) ? clock64() : 0;
-    if (g == 0 && (pf & F_M0)) {
-      const u32* m = c->p_m[0];
-      grp_split<K, V>(gt, T.BK(m[0]), T.BV(m[0]), K, T.BK(m[1]), T.BV(m[1]), K, K, T.BK(m[2]), T.BV(m[2]),
-                      T.BK(m[3]), T.BV(m[3]), mwin);
-    }
-    if (g == 1 && (pf & F_M1)) {
-      const u32* m = c->p_m[1];
-      grp_split<K, V>(gt, T.BK(m[0]), T.BV(m[0]), K, T.BK(m[1]), T.BV(m[1]), K, K, T.BK(m[2]), T.BV(m[2]),
-                      T.BK(m[3]), T.BV(m[3]), mwin);
-    }
-    if (g == 2 && (pf & F_LAG) && !(pf & F_LAGDONE)) {
-      mbar_wait(&c->sbar[w_sbi], w_spar);
-      if (c->stg_st[w_sbi][0] == ST_AVAIL && c->stg_st[w_sbi][1] == ST_AVAIL) {
-        const u32* m = c->p_m[2];
-        grp_split<K, V>(gt, T.BK(m[0]), T.BV(m[0]), K, T.BK(m[1]), T.BV(m[1]), K, K, T.BK(m[2]), T.BV(m[2]),
-                        T.BK(m[3]), T.BV(m[3]), mwin);
-      }
-    }
-    if (lt && gt == 0) c->tm[8 + g] += clock64() - ta;
-    // the TMA data the control warp reads next (staged children, refill node) has landed
-    const ull tw = (lt && gt == 0) ? clock64() : 0;
-    if (pf & F_LAG) mbar_wait(&c->sbar[w_sbi], w_spar);
-    if (w_rwait) mbar_wait(&c->rbar[w_rbi], w_rpar);
-    if (lt && gt == 0) c->tm[3] += clock64() - tw;
-    nbar_arrive(DT_BAR_DONE, NB_);
-  }
-}
-
-// control warp, lane 0 works; the whole warp takes part in the named barriers
-template <int K, bool V>
-__device__ __forceinline__ void dt_control(DTop<K, V>& T) {
-  DtCtl* c = T.c;
-  const HeapArgs& H = T.H;
-  const CallArgs& C = T.C;
-  const u32 lane = threadIdx.x & 31;
-  const u64 n_ops = C.n_ops;
-  constexpr u32 NBY = K * 4u;
-  constexpr int NB_ = DT_NTC + 32;
-  DtS& SS = c->s;
-  if (lane == 0) {
-    DtS* __restrict__ const Sp = &SS;
-    DtS& S = *Sp;
-    S.init();
-    S.fm = (1u << DT_NSLOT) - 1u;
-    S.defer = 1;
-    S.hs = ld_relaxed(H.hdr + H_HS);
-    S.rs = ld_relaxed(H.hdr + H_RS);
-    S.ps = ld_relaxed(H.hdr + H_PS);
-    u32 bytes = 0;
-    for (u32 q = 0; q < 8; ++q) {
-      const bool have = q == 0 ? S.ps > 0 : (q == 1 ? (S.hs >= 1 && S.rs > 0) : q <= S.hs);
-      c->ns[q] = have ? T.alloc(S) : DT_NONE;
-      if (have) bytes += V ? 2u * NBY : NBY;
-    }
-    fence_proxy_async();
-    mbar_arrive_expect_tx(&c->lbar, bytes);
-    for (u32 q = 0; q < 8; ++q) {
-      if (c->ns[q] == DT_NONE) continue;
-      bulk_g2s(T.BK(c->ns[q]), H.gk + (size_t)q * K, NBY, &c->lbar);
-      if (V) bulk_g2s(T.BV(c->ns[q]), H.gv + (size_t)q * K, NBY, &c->lbar);
-    }
-    mbar_wait(&c->lbar, 0);
-    dt_plan<K, V>(T, S, n_ops, false);
-  }
-  __syncwarp();
-  const bool lt = (C.debug & 128u) != 0;
-  ull t0 = lt ? clock64() : 0, t1 = 0;
-  for (;;) {
-    if (*reinterpret_cast<volatile u32*>(&c->p_flags) == DT_NONE) break;
-    if (lt && lane == 0) { t1 = clock64(); c->tm[0] += t1 - t0; c->tm[5]++; }  // decisions (+ plan)
-    nbar_arrive(DT_BAR_READY, NB_);  // the groups run phase A of this slot
-    if (lane == 0) {
-      DtS* __restrict__ const Sp = &SS;
-    DtS& S = *Sp;
-      T.flush(S);  // helper requests of the decisions just taken and of the plan
-      // Alg.2 l.18-22: the old root keys are the first output of op i (TMA bulk store)
-      if (c->p_flags & F_NEW) {
-        const u32 n = c->p_out_n;
-        if (n) {
-          const u64 pos0 = (((u64)c->p_iop_hi << 32) | c->p_iop_lo) * (u64)K;
-          const u32 src = c->p_out_slot;
-          const bool bulk = (n & 3u) == 0 && ((reinterpret_cast<uintptr_t>(C.out_k + pos0) & 15u) == 0) &&
-                            (!V || !C.out_v || (reinterpret_cast<uintptr_t>(C.out_v + pos0) & 15u) == 0);
-          if (bulk) {
-            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-            bulk_s2g(C.out_k + pos0, T.BK(src), n * 4u);
-            if (V && C.out_v) bulk_s2g(C.out_v + pos0, T.BV(src), n * 4u);
-            asm volatile("cp.async.bulk.commit_group;" ::: "memory");
-          } else {
-            for (u32 q = 0; q < n; ++q) {
-              C.out_k[pos0 + q] = T.BK(src)[q];
-              if (V && C.out_v) C.out_v[pos0 + q] = T.BV(src)[q];
-            }
-          }
-        }
-      }
-    }
-    __syncwarp();
-    if (lt && lane == 0) { const ull t = clock64(); c->tm[2] += t - t1; t1 = t; }  // flush + output copy
-    nbar_sync(DT_BAR_DONE, NB_);  // phase A done, staged / refill data visible
-    if (lt && lane == 0) { t0 = clock64(); c->tm[1] += t0 - t1; }  // waiting for phase A
-    if (lane == 0) SS.stage = 0;
-    for (;;) {
-      if (lane == 0) {
-        DtS* __restrict__ const Sp = &SS;
-        DtS& S = *Sp;
-        c->njobs = 0;
-        bool done = false;
-        if (S.stage == 0) done = dt_fast<K, V>(T, S);
-        if (!done) done = dt_slow<K, V>(T, S, false);
-        if (done) dt_plan<K, V>(T, S, n_ops, false);
-        else c->p_flags = F_JOBS;
-        c->ctl_done = done ? 1u : 0u;
-      }
-      __syncwarp();
-      if (*reinterpret_cast<volatile u32*>(&c->ctl_done)) break;
-      nbar_arrive(DT_BAR_READY, NB_);  // the groups run the job list
-      nbar_sync(DT_BAR_DONE, NB_);
-    }
-  }
-  // ---- call end: the on-chip part back to the arena (a job list for the groups)
-  if (lane == 0) {
-    DtS* __restrict__ const Sp = &SS;
-    DtS& S = *Sp;
-    T.flush(S);
-    c->njobs = 0;
-    for (u32 q = 0; q < 8; ++q) {
-      const u32 sl = c->ns[q];
-      if (q >= 1) st_relaxed(T.stp(q), q <= S.hs ? ST_AVAIL : ST_EMPTY);
-      if (sl == DT_NONE) continue;
-      const u32 cnt = q == 0 ? S.ps : (q == 1 ? S.rs : K);
-      if (q > S.hs || cnt == 0) continue;
-      st_relaxed(&H.meta[q].kmin, T.BK(sl)[0]);
-      st_relaxed(&H.meta[q].kmax, T.BK(sl)[cnt - 1]);
-      T.job(J_STORE, q, sl);
-    }
-    c->p_flags = F_JOBS;
-  }
-  __syncwarp();
-  nbar_arrive(DT_BAR_READY, NB_);
-  nbar_sync(DT_BAR_DONE, NB_);
-  if (lane == 0) {
-    DtS* __restrict__ const Sp = &SS;
-    DtS& S = *Sp;
-    st_relaxed(H.hdr + H_HS, S.hs);
-    st_relaxed(H.hdr + H_RS, S.rs);
-    st_relaxed(H.hdr + H_PS, S.ps);
-    ull lin;
-    asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(lin) : "l"(H.hdr + H_LIN) : "memory");
-    asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(H.hdr + H_LIN), "l"(lin + n_ops) : "memory");
-    c->st[S_KEYS_OUT] += S.nout;
-    if (C.d_count && S.nout) atomicAdd(C.d_count, (ull)S.nout);
-    asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
-    T.enqueue(RQ_END);
-    T.enqueue(RQ_STAGE, 0u, 0u, 0u, 0u, DT_NONE);
-    while (ld_acq_cta(&c->rq_done[0]) != c->rq_head[0] || ld_acq_cta(&c->rq_done[1]) != c->rq_head[1]) {}
-    ull* stat = reinterpret_cast<ull*>(H.hdr + H_STAT);
-    for (int q = 0; q < NSTAT; ++q)
-      if (c->st[q]) atomicAdd(stat + q, c->st[q]);
-    if (lt) {
-      ull* tms = reinterpret_cast<ull*>(H.hdr + H_TIME);
-      for (int q = 0; q < 12; ++q) { atomicAdd(tms + 16 + q, c->tm[q]); atomicAdd(tms + q, c->ts[q]); }
-    }
-    c->p_flags = DT_NONE;
-  }
-  __syncwarp();
-  nbar_arrive(DT_BAR_READY, NB_);  // the groups leave
-}
-
 // =========================================================================================
 // Walkers: Alg.3 from l.2 at a depth-3 node handed over by the top CTA (locked, carried
 // keys stored in the node), with OpL's lock-ahead agents (bgpq_locks.cuh).
@@ -1603,18 +1397,13 @@ __global__ void __launch_bounds__(DT_BLOCK, 1) bgpq_dtop_kernel(HeapArgs H, Call
       asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     __syncthreads();
-    const bool ctlw = (C.debug & 512u) != 0;  // test switch 512: the control-warp driver (dt_control)
     if (threadIdx.x >= DT_NTC + 32) {
       if (threadIdx.x == DT_NTC + 32) dt_helper<K, V>(T, 0u);
       if (threadIdx.x == DT_NTC + 64) dt_helper<K, V>(T, 1u);
       return;
     }
-    if (threadIdx.x >= DT_NTC) {
-      if (ctlw) dt_control<K, V>(T);
-      return;
-    }
-    if (ctlw) dt_groups2<K, V>(T);
-    else dt_top<K, V>(T);
+    if (threadIdx.x >= DT_NTC) return;  // control warp: idle
+    dt_top<K, V>(T);
     return;
   }
   // ---- walkers

@@ -968,6 +968,13 @@ __global__ void __launch_bounds__(NT + 32, 1) bgpq_locks_kernel(HeapArgs H, Call
       ins = C.op_types[j] == 0;
       size = C.op_sizes[j];
       lt = C.lin_ticket ? C.lin_ticket + j : nullptr;
+      if (size == 0u || size > (u32)K) {  // op sizes must be in 1..K: sticky EINVAL, op skipped
+        if (threadIdx.x == 0) {
+          atomicCAS(H.hdr + H_ERR, 0u, (u32)-1);
+          if (!ins) C.op_count[j] = 0;
+        }
+        continue;
+      }
       if (ins) {
         const u64 off = C.in_off[j];
         ik = C.in_k + off;

@@ -320,40 +320,4 @@ struct Pipe {
   }
 };
 
-template <int K, bool V, int NT>
-__global__ void __launch_bounds__(NT, 1) bgpq_ins_pipe_kernel(HeapArgs H, PipeArgs P, CallArgs C) {
-  extern __shared__ __align__(128) unsigned char smem_raw[];
-  LCtl* ctl = reinterpret_cast<LCtl*>(smem_raw);
-  Pipe<K, V, NT> p;
-  p.H = H;
-  p.P = P;
-  p.C = C;
-  p.ctl = ctl;
-  p.sk = reinterpret_cast<u32*>(smem_raw + LCTL_BYTES);
-  p.sv = p.sk + 6 * K;
-  p.ph0 = 0;
-  p.ph1 = 0;
-  if (threadIdx.x == 0) {
-    mbar_init(&ctl->bar, 1);
-    for (int i = 0; i < NSTAT; ++i) ctl->st[i] = 0;
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-  }
-  __syncthreads();
-  const u32 b = blockIdx.x;
-  if (b == 0) p.root_stage();
-  else if (b <= P.depth) p.level_stage(b);
-  else p.sorter();
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    ull* stat = reinterpret_cast<ull*>(H.hdr + H_STAT);
-    for (int i = 0; i < NSTAT; ++i)
-      if (ctl->st[i]) atomicAdd(stat + i, ctl->st[i]);
-  }
-}
-
-template <int K, bool V>
-constexpr size_t pipe_smem_bytes() {
-  return LCTL_BYTES + (size_t)6 * K * 4 * (V ? 2 : 1);
-}
-
 }  // namespace bgpqd

@@ -35,8 +35,11 @@ def _inv(q):
     return oracle.check_invariants(q.K, q.slots() - 1, h["heapSize"], h["rootSize"], h["pbSize"], nk, states)
 
 
-@pytest.mark.parametrize("K,values", [(64, True), (128, False), (1024, True), (1024, False)])
-def test_call_sequence_vs_oracle(K, values):
+@pytest.mark.parametrize("K,values,dist", [(64, True, "uniform"), (128, False, "uniform"), (512, False, "uniform"),
+                                           (512, True, "uniform"), (1024, True, "uniform"),
+                                           (1024, False, "uniform"), (256, False, "gaussian"),
+                                           (1024, False, "gaussian"), (512, True, "gaussian")])
+def test_call_sequence_vs_oracle(K, values, dist):
     """Random insert / deletemin calls of ragged sizes on one heap, call by call vs the oracle:
     crosses the pipelined / synchronous boundary (heapSize 64) in both directions, drains to
     empty (|root| = 0 afterwards) and refills."""
@@ -51,7 +54,7 @@ def test_call_sequence_vs_oracle(K, values):
             ("del", 600 * K), ("ins", 90 * K + 33), ("del", 45 * K), ("del", 600 * K)]
     for kind, n in plan:
         if kind == "ins":
-            keys = synth.keys(n, seed=int(rng.integers(1 << 30)))
+            keys = synth.keys(n, seed=int(rng.integers(1 << 30)), dist=dist)
             keys = (keys % np.uint32(1 << 20)).astype(np.uint32) if K == 128 else keys  # duplicates
             vals = np.arange(base, base + n, dtype=np.uint32)
             base += n

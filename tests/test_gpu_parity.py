@@ -33,13 +33,13 @@ def _gpu_inv(q):
 # --------------------------------------------------------------------------------------
 # phased insert-all then deletemin-all: output == sorted(input) (closed form, §8(c))
 # --------------------------------------------------------------------------------------
-MODES = ["default", "locks", "server"]
+MODES = ["default", "locks"]
 
 
 def _mode(mode):
     """default: INSERT calls as the level pipeline + top-CTA DELETEMIN with walkers; locks: paper-literal
-    per-node locks for every call; server: root-server execution."""
-    return {"locks": mode == "locks", "server": mode == "server"}
+    per-node locks for every call."""
+    return {"locks": mode == "locks"}
 
 
 @pytest.mark.parametrize("mode", MODES)
@@ -47,8 +47,6 @@ def _mode(mode):
 @pytest.mark.parametrize("dist", ["uniform", "ascending", "descending", "gaussian", "dups"])
 def test_phased_sorted(K, dist, mode):
     n = 40 * K + 37  # several tiles and a ragged tail
-    if mode == "server":
-        n = 300 * K + 37  # deeper than the on-chip levels for every K
     keys = synth.keys(n, seed=synth.SEEDS["C3"], dist=dist)
     vals = synth.values(n)
     q = pkg.BGPQ(capacity=n, K=K, values=True, **_mode(mode))
@@ -62,6 +60,49 @@ def test_phased_sorted(K, dist, mode):
     assert np.array_equal(np.sort(outv), np.arange(n, dtype=np.uint32))
     assert q.size() == 0
     q.close()
+
+
+@pytest.mark.parametrize("values", [False, True])
+@pytest.mark.parametrize("K", [64, 128, 256, 512, 1024])
+@pytest.mark.parametrize("dist", ["uniform", "ascending", "descending", "gaussian", "dups"])
+def test_phased_sorted_pipelined(K, dist, values):
+    """heapSize >= 64 (300 nodes): the top CTA runs its pipelined mode (refill taken one slot
+    ahead, depths 0-2 on chip, walkers below) for most of the drain; keys-only at K >= 512 takes
+    the bitonic SORT_SPLIT in the insert pipeline, the top CTA's groups and the walkers."""
+    n = 300 * K + 17
+    keys = synth.keys(n, seed=synth.SEEDS["C3"] + K, dist=dist)
+    q = pkg.BGPQ(capacity=n, K=K, values=values)
+    q.insert(_dev(keys), _dev(synth.values(n)) if values else None)
+    assert q.size() == n
+    ok, ov = q.deletemin(n)
+    outk = _host(ok)
+    assert np.array_equal(outk, np.sort(keys))
+    if values:
+        outv = _host(ov)
+        assert np.array_equal(keys[outv], outk)
+        assert np.array_equal(np.sort(outv), np.arange(n, dtype=np.uint32))
+    assert q.size() == 0
+    q.close()
+
+
+@pytest.mark.parametrize("dist", ["uniform", "ascending", "descending", "gaussian"])
+def test_c3_matrix_full_size(dist):
+    """Config C3 in full (BASELINE configs[2]): 2^26 keys of each distribution at K in
+    {128, 256, 512, 1024}, keys only, phased insert-all / deletemin-all on one handle per K;
+    the concatenated output must equal sorted(input) (closed form, §8(c))."""
+    n = 1 << 26
+    keys = synth.keys(n, seed=synth.SEEDS["C3"], dist=dist)
+    srt = np.sort(keys)
+    dk = _dev(keys)
+    for K in (128, 256, 512, 1024):
+        q = pkg.BGPQ(capacity=n, K=K, values=False)
+        q.insert(dk)
+        assert q.size() == n
+        ok, _ = q.deletemin(n)
+        assert np.array_equal(_host(ok), srt), (dist, K)
+        assert q.size() == 0
+        q.close()
+        del ok
 
 
 def test_phased_c1_keys_only():
@@ -94,6 +135,16 @@ def _compare_layout(q, seq):
     assert np.array_equal(nk[live], sk[live])
 
 
+def _compare_counters(q, seq, before=None):
+    """Device counters (bench.py's byte model) equal the sequential model's counters."""
+    g = q.stats()
+    if before is not None:
+        g = {k: g[k] - before[k] for k in g}
+    g["del_lr_merge"] += g["del_lr_nomove"]  # the GPU splits l/r SORT_SPLITs into moving / no-move
+    for k, v in seq.counters().items():
+        assert g[k] == v, (k, g[k], v)
+
+
 @pytest.mark.parametrize("K", [64, 256])
 def test_serialized_layout_bitexact_phased(K):
     n = 96 * K + 5
@@ -109,9 +160,10 @@ def test_serialized_layout_bitexact_phased(K):
     want = np.concatenate([seq.deletemin(K)[0] for _ in range(37)])
     assert np.array_equal(_host(ok), want)
     _compare_layout(q, seq)
+    _compare_counters(q, seq)
 
 
-@pytest.mark.parametrize("K", [64, 1024])
+@pytest.mark.parametrize("K", [64, 512, 1024])
 @pytest.mark.parametrize("values", [False, True])
 def test_pipelined_insert_layout_bitexact(K, values):
     """INSERT calls run as a level pipeline that applies the batches at every node in call
@@ -181,19 +233,24 @@ def test_serialized_mixed_partial_sizes_bitexact():
 # concurrent mixes: replay the linearization log (ticket order) through the oracle
 # --------------------------------------------------------------------------------------
 def _replay_check(types, sizes, keys, in_off, outk, outv, cnt, lin, prefill=None):
+    """Ticket-order replay (the linearization point is in the root section) through
+    oracle.replay: every deletemin's keys bit-exact.  Returns the oracle queue after the log."""
     order = np.argsort(lin, kind="stable")
     assert np.array_equal(lin[order], np.arange(len(lin)) + (lin.min() if len(lin) else 0))
-    q = oracle.OraclePQ()
-    if prefill is not None:
-        q.insert(prefill)
+    log = [] if prefill is None else [(0, (prefill, None))]
     for j in order:
         if types[j] == 0:
-            q.insert(keys[in_off[j]:in_off[j] + sizes[j]])
+            log.append((0, (keys[in_off[j]:in_off[j] + sizes[j]], None)))
         else:
-            want, _ = q.deletemin(int(sizes[j]))
-            got = outk[j, :cnt[j]]
-            assert cnt[j] == len(want), f"op {j}: count {cnt[j]} != {len(want)}"
-            assert np.array_equal(got, want), f"op {j} (ticket {lin[j]}) differs from replay"
+            log.append((1, int(sizes[j])))
+    q = oracle.OraclePQ()
+    res = oracle.replay(log, q=q)
+    dels = [j for j in order if types[j] == 1]
+    assert len(res) == len(dels)
+    for j, (want, _) in zip(dels, res):
+        got = outk[j, :cnt[j]]
+        assert cnt[j] == len(want), f"op {j}: count {cnt[j]} != {len(want)}"
+        assert np.array_equal(got, want), f"op {j} (ticket {lin[j]}) differs from replay"
     return q
 
 
@@ -250,6 +307,8 @@ def test_marked_handoff_replay(mode):
         assert _gpu_inv(q) == (0, 0)
         total_marked += q.stats()["marked"]
     print("MARKED hand-offs observed:", total_marked)
+    if mode == "locks":  # every call on the per-node-lock engine: the collaboration must fire
+        assert total_marked > 0
 
 
 # --------------------------------------------------------------------------------------

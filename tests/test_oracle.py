@@ -341,3 +341,74 @@ def test_seq_model_sorted_input_special_cases(K):
     assert _check_inv(q) == (0, 0)
     out = np.concatenate([q.deletemin(K)[0] for _ in range(nb)])
     assert np.array_equal(out, base)
+
+
+def test_replay_matches_bruteforce_log():
+    """oracle.replay (used by the GPU ticket-order replays) against a brute-force sorted list
+    on random logs with partial sizes and over-asking deletemins (fewer than asked ->
+    everything left; x_{k+1} = min_r(I_k - D_k))."""
+    rng = np.random.default_rng(5)
+    for trial in range(30):
+        log, brute, want = [], [], []
+        for _ in range(60):
+            if rng.random() < 0.55:
+                k = rng.integers(0, 40, rng.integers(1, 9)).astype(np.uint32)
+                log.append((0, (k, None)))
+                brute.extend(int(x) for x in k)
+            else:
+                m = int(rng.integers(1, 12))
+                log.append((1, m))
+                brute.sort()
+                want.append(brute[:m])
+                del brute[:m]
+        got = oracle.replay(log)
+        assert len(got) == len(want)
+        for (gk, _), w in zip(got, want):
+            assert gk.tolist() == w
+    q = oracle.OraclePQ()
+    oracle.replay([(0, (np.array([3, 1, 2], np.uint32), None)), (1, 2)], q=q)
+    assert q.size() == 1 and q.deletemin(5)[0].tolist() == [3]
+
+
+def test_invariant_checker_root_and_buffer_codes():
+    """Codes -5 (pBuffer entry below the root's max: P:146 keeps every buffered key >= the
+    root's keys) and -6 (non-empty heap whose root is not AVAIL)."""
+    K = 4
+    q = oracle.SeqBGPQ(K, 32)
+    keys = synth.keys(4 * 6 + 2, seed=12)
+    for off in range(0, 24, 4):
+        q.insert(keys[off:off + 4])
+    q.insert(keys[24:26])                      # partial batch -> pBuffer non-empty
+    h = q.header()
+    assert h["pbSize"] > 0 and h["rootSize"] == K
+    nk, _, st = q.dump()
+    args = (K, q.cap, h["heapSize"], h["rootSize"], h["pbSize"])
+    assert oracle.check_invariants(*args, nk, st) == (0, 0)
+    bad = nk.copy(); bad[0][0] = 0; bad[1][:] = np.sort(bad[1]); bad[0][:h["pbSize"]].sort()
+    bad[1][K - 1] = 0xFFFFFFFF                 # root max above the buffer's min
+    assert oracle.check_invariants(*args, bad, st)[0] == -5
+    bad_st = st.copy(); bad_st[1] = oracle.EMPTY
+    assert oracle.check_invariants(*args, nk, bad_st)[0] == -6
+
+
+def test_seq_model_del_levels_closed_forms():
+    """DELETEMIN_HEAPIFY level counter (the byte model's del_levels, Alg.3 l.4): with all keys
+    equal, l.4's stop test max(cur) <= min(l, r) holds at the root, so no level is traversed and
+    every full-K deletemin but the last refills (Alg.2 l.5-14); with two batches the single
+    refill walks at most one level (root -> node 2 has no children)."""
+    K, nb = 8, 50
+    q = oracle.SeqBGPQ(K, nb + 2)
+    for _ in range(nb):
+        q.insert(np.full(K, 9, np.uint32))
+    for _ in range(nb):
+        assert q.deletemin(K)[0].tolist() == [9] * K
+    c = q.counters()
+    assert c["del_levels"] == 0 and c["del_ops"] == nb and c["del_refill_ops"] == nb - 1
+    q = oracle.SeqBGPQ(K, 8)
+    q.insert(np.arange(8, 16, dtype=np.uint32))
+    q.insert(np.arange(0, 8, dtype=np.uint32))
+    q.insert(np.arange(16, 24, dtype=np.uint32))  # heapSize 3: root [0..7], node 2 [8..15], node 3 [16..23]
+    assert q.deletemin(K)[0].tolist() == list(range(8))
+    c = q.counters()
+    # refill takes node 3 into the root; one level: l = 2 AVAIL, r = 3 now EMPTY (R5) -> y = 2
+    assert c["del_refill_ops"] == 1 and c["del_levels"] == 1 and c["del_lr_skip"] == 1

@@ -1,7 +1,8 @@
-"""Top-CTA timers of the deletemin execution: BGPQ_DEBUG=8 python tools/dt_timers.py [lg] [K]"""
+"""Top-CTA timers of the deletemin execution: python tools/dt_timers.py [lg] [K]"""
 import sys, numpy as np, torch
 sys.path.insert(0, ".")
 import synth, paper_conf_icpp_chenhjz21_b200 as pkg
+pkg.set_debug(8)
 lg = int(sys.argv[1]) if len(sys.argv) > 1 else 24
 K = int(sys.argv[2]) if len(sys.argv) > 2 else 1024
 n = 1 << lg
@@ -11,7 +12,7 @@ dk = torch.from_numpy(keys.view(np.int32)).cuda()
 out = torch.empty(n, dtype=torch.int32, device="cuda")
 def raw():
     o = np.zeros(32, np.uint64)
-    pkg.lib().bgpq_timers(q._h, o.ctypes.data_as(pkg._vp))
+    o[:] = q.timers()
     return o.astype(np.float64)
 q.insert(dk); torch.cuda.synchronize()
 t1 = raw()

@@ -1,7 +1,8 @@
-"""Per-level INSERT pipeline timers: BGPQ_DEBUG=128 python tools/pipe_timers.py [lg]"""
+"""Per-level INSERT pipeline timers: python tools/pipe_timers.py [lg]"""
 import sys, numpy as np, torch
 sys.path.insert(0, ".")
 import synth, paper_conf_icpp_chenhjz21_b200 as pkg
+pkg.set_debug(128)
 lg = int(sys.argv[1]) if len(sys.argv) > 1 else 27
 n = 1 << lg
 keys = synth.keys(n, seed=2)
@@ -9,7 +10,7 @@ q = pkg.BGPQ(capacity=n, K=1024, values=False)
 dk = torch.from_numpy(keys.view(np.int32)).cuda()
 e = [torch.cuda.Event(enable_timing=True) for _ in range(2)]
 e[0].record(); q.insert(dk); e[1].record(); torch.cuda.synchronize()
-o = np.zeros(32, np.uint64); pkg.lib().bgpq_timers(q._h, o.ctypes.data_as(pkg._vp))
+o = np.zeros(32, np.uint64); o[:] = q.timers()
 print("insert ms %.1f  (cycles, Mcyc)" % e[0].elapsed_time(e[1]))
 levels = list(range(1, 10)) + [14, 15, 16]
 for idx, l in enumerate(levels):
