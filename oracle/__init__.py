@@ -19,6 +19,7 @@ import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _SRC = os.path.join(_HERE, "bgpq_oracle.cpp")
+_SRCS = [_SRC, os.path.join(_HERE, "apps_oracle.cpp")]
 _LIB = os.path.join(_HERE, "liboracle.so")
 
 AVAIL, EMPTY, TARGET, MARKED = 0, 1, 2, 3  # P:180 §4
@@ -30,8 +31,8 @@ _i64p = ctypes.POINTER(ctypes.c_longlong)
 
 def build(force: bool = False) -> str:
     """Compile liboracle.so with g++ (-O2, C++17).  Building the checker is not using it."""
-    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
-        cmd = ["g++", "-O2", "-std=c++17", "-shared", "-fPIC", "-o", _LIB + ".tmp", _SRC]
+    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < max(map(os.path.getmtime, _SRCS)):
+        cmd = ["g++", "-O2", "-std=c++17", "-shared", "-fPIC", "-o", _LIB + ".tmp", *_SRCS]
         subprocess.check_call(cmd)
         os.replace(_LIB + ".tmp", _LIB)
     return _LIB
@@ -70,6 +71,12 @@ def lib():
         L.orc_check_invariants.argtypes = [ctypes.c_uint32, ctypes.c_uint32, ctypes.c_uint32,
                                            ctypes.c_uint32, ctypes.c_uint32, _u32p, _u32p, _u64p]
         L.orc_check_invariants.restype = ctypes.c_int
+        for nm in ("orc_ks_dp", "orc_ks_brute"):
+            getattr(L, nm).argtypes = [ctypes.c_uint32, _u32p, _u32p, ctypes.c_uint64]
+            getattr(L, nm).restype = ctypes.c_longlong
+        L.orc_ks_bnb.argtypes = [ctypes.c_uint32, _u32p, _u32p, ctypes.c_uint64, _u64p]
+        for nm in ("orc_astar", "orc_dijkstra"):
+            getattr(L, nm).argtypes = [ctypes.c_uint32, ctypes.c_uint32, ctypes.c_void_p] + [ctypes.c_uint32] * 4 + [_u64p]
         _lib = L
     return _lib
 
@@ -212,3 +219,56 @@ def replay(ops, q=None):
         else:
             res.append(q.deletemin(int(payload)))
     return res
+
+
+# ---------------------------------------------------------------------------------------
+# applications (apps_oracle.cpp)
+# ---------------------------------------------------------------------------------------
+UNREACHABLE = (1 << 64) - 1
+
+
+def ks_dp(w, p, C) -> int:
+    """0-1 knapsack optimum by the textbook dynamic program (pin)."""
+    w, p = _u32(w), _u32(p)
+    r = lib().orc_ks_dp(len(w), _p32(w), _p32(p), int(C))
+    if r < 0:
+        raise ValueError("capacity too large for the DP")
+    return int(r)
+
+
+def ks_brute(w, p, C) -> int:
+    """0-1 knapsack optimum by enumerating every subset, n <= 24 (pin)."""
+    w, p = _u32(w), _u32(p)
+    r = lib().orc_ks_brute(len(w), _p32(w), _p32(p), int(C))
+    if r < 0:
+        raise ValueError("n > 24")
+    return int(r)
+
+
+def ks_bnb(w, p, C) -> dict:
+    """Sequential best-first branch and bound (readings R23): optimum, nodes
+    expanded, nodes inserted into the priority queue."""
+    w, p = _u32(w), _u32(p)
+    out = (ctypes.c_uint64 * 3)()
+    lib().orc_ks_bnb(len(w), _p32(w), _p32(p), int(C), out)
+    return {"optimum": int(out[0]), "expanded": int(out[1]), "inserted": int(out[2])}
+
+
+def _grid_call(fn, grid, src, dst):
+    g = np.ascontiguousarray(grid, dtype=np.uint8)
+    N, M = g.shape
+    out = (ctypes.c_uint64 * 2)()
+    fn(N, M, g.ctypes.data_as(ctypes.c_void_p), int(src[0]), int(src[1]), int(dst[0]), int(dst[1]), out)
+    return int(out[0]), int(out[1])
+
+
+def astar(grid, src, dst) -> dict:
+    """Sequential A* (reading R24: 8 moves, orthogonal 1 / diagonal 2, Manhattan h):
+    shortest path cost (UNREACHABLE if none) and nodes expanded."""
+    c, e = _grid_call(lib().orc_astar, grid, src, dst)
+    return {"cost": c, "expanded": e}
+
+
+def dijkstra(grid, src, dst) -> int:
+    """Dijkstra on the same graph (pin of the A* cost)."""
+    return _grid_call(lib().orc_dijkstra, grid, src, dst)[0]
