@@ -131,6 +131,23 @@ int bgpq_grid(bgpq_t* q);
 /* Number of kernels this library has launched in the process (for bench gpu_launches). */
 uint64_t bgpq_launch_count(void);
 
+/* Device view of a heap for application kernels that call the device API
+ * (include/bgpq_dev.cuh): plain device pointers of the arena owned by the handle (valid until
+ * bgpq_destroy), the node capacity, K, the creation flags, the device and its SM count.  No
+ * library call may run on the heap while such a kernel does. */
+typedef struct {
+  void* keys;     /* uint32 node keys, slot i at keys + i*K (0 = pBuffer, 1 = root) */
+  void* vals;     /* uint32 node values, same layout, or NULL for a keys-only heap   */
+  void* meta;     /* 16-B node records {lock, state, min, max}, one per slot          */
+  void* hdr;      /* header words                                                     */
+  uint32_t cap;   /* largest node index                                               */
+  uint32_t K;
+  uint32_t flags;
+  int device;
+  int sm_count;
+} bgpq_view_t;
+int bgpq_view(bgpq_t* q, bgpq_view_t* out);
+
 /* Test / profiling extensions (not part of the minimal ABI).
  * bgpq_set_debug: process-wide switches read at each call (0 = product behaviour):
  *   8   accumulate thread-0 cycle timers in the header (read with bgpq_timers);

@@ -36,7 +36,8 @@ VALID_K = (64, 128, 256, 512, 1024)
 
 
 def _sources():
-    return [os.path.join(_CSRC, f) for f in sorted(os.listdir(_CSRC))] + [os.path.join(_INCLUDE, "bgpq.h")]
+    return [os.path.join(_CSRC, f) for f in sorted(os.listdir(_CSRC))] + \
+        [os.path.join(_INCLUDE, f) for f in sorted(os.listdir(_INCLUDE))]
 
 
 def build(force: bool = False, verbose: bool = False, jobs: int | None = None) -> str:
@@ -51,6 +52,7 @@ def build(force: bool = False, verbose: bool = False, jobs: int | None = None) -
               os.path.join(BUILD_DIR, f"kern_{k}_{v}.o")) for k, v in KERNEL_UNITS]
     units.append(([], os.path.join(_CSRC, "bgpq_api.cu"), os.path.join(BUILD_DIR, "api.o")))
     units.append(([], os.path.join(_CSRC, "bgpq_testprim.cu"), os.path.join(BUILD_DIR, "testprim.o")))
+    units.append(([], os.path.join(_CSRC, "bgpq_apps.cu"), os.path.join(BUILD_DIR, "apps.o")))
     jobs = jobs or max(1, min(len(units), os.cpu_count() or 1))
     pending, running, logs = list(units), [], []
     while pending or running:

@@ -448,6 +448,20 @@ int bgpq_set_grid(bgpq_t* q, int ctas) {
 
 int bgpq_grid(bgpq_t* q) { return q ? grid_for(q, ~0ull) : 0; }
 
+int bgpq_view(bgpq_t* q, bgpq_view_t* out) {
+  if (!q || !out) return fail(BGPQ_EINVAL);
+  out->keys = q->gk;
+  out->vals = (q->flags & BGPQ_FLAG_VALUES) ? q->gv : nullptr;
+  out->meta = q->meta;
+  out->hdr = q->hdr;
+  out->cap = q->cap_nodes;
+  out->K = q->K;
+  out->flags = q->flags;
+  out->device = q->device;
+  out->sm_count = q->sm_count;
+  return BGPQ_OK;
+}
+
 int bgpq_set_debug(uint32_t bits) {
   g_debug = bits;
   return BGPQ_OK;
