@@ -100,6 +100,24 @@ struct Queue {
     if (threadIdx.x == 0) op.st[bgpqd::S_KEYS_OUT] += r;
     return r;
   }
+  // Approximate number of keys in the heap from the header words, read without the root
+  // lock (a hint: exact at quiescence).  Identical in every compute thread.  Lets a CTA that
+  // would only find an empty heap back off instead of taking the root lock away from
+  // the CTAs that are inserting.
+  __device__ __forceinline__ u64 size_hint() {
+    sync();
+    if (threadIdx.x == 0) {
+      const u32 hs = bgpqd::ld_relaxed(op.H.hdr + bgpqd::H_HS);
+      const u32 rs = bgpqd::ld_relaxed(op.H.hdr + bgpqd::H_RS);
+      const u32 ps = bgpqd::ld_relaxed(op.H.hdr + bgpqd::H_PS);
+      const u64 n = hs == 0 ? 0ull : (u64)rs + ps + (u64)(hs - 1) * K;
+      op.ctl->b[22] = n > 0xFFFFFFFFull ? 0xFFFFFFFFu : (u32)n;
+    }
+    sync();
+    const u64 r = op.ctl->b[22];
+    sync();
+    return r;
+  }
   // Compute threads: stop the lock warp and add this CTA's device counters to the heap's.
   __device__ __forceinline__ void finish() {
     sync();

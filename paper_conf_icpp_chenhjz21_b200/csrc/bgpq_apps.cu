@@ -107,6 +107,7 @@ struct KsSmem {
   u32 chk[2 * K], chv[2 * K];
   u32 warp_tot[32];
   u32 total;
+  u32 done;
 };
 
 template <int K>
@@ -123,14 +124,21 @@ __global__ void __launch_bounds__(ANT + 32, 1)
   KsSmem<K>& S = *reinterpret_cast<KsSmem<K>*>(smem_raw + Q::smem_bytes());
   const int tid = threadIdx.x;
   ull expanded = 0, inserted = 0, pops = 0, pruned = 0, empty = 0;
+  u32 backoff = 128;
   for (u32 it = 0; it < budget; ++it) {
-    const u32 c = q.deletemin(S.popk, S.popv, K);
-    if (c == 0) {
+    const u32 c = q.size_hint() ? q.deletemin(S.popk, S.popv, K) : 0u;
+    if (c == 0) {  // nothing in the heap: done if nothing is in flight either (uniform decision)
       ++empty;
-      if (ld_acq64(state + ST_PENDING) == 0) break;
-      __nanosleep(256);
+      if (tid == 0) S.done = ld_acq64(state + ST_PENDING) == 0;
+      cta_bar<ANT>();
+      const bool done = S.done;
+      cta_bar<ANT>();
+      if (done) break;
+      __nanosleep(backoff);
+      backoff = backoff < 8192 ? backoff * 2 : 8192;
       continue;
     }
+    backoff = 128;
     ++pops;
     const ull inc = ld_acq64(state + ST_INC);
     // expand: thread t handles popped node t (K <= ANT * 2: two rounds at K = 1024)
@@ -268,6 +276,7 @@ struct AsSmem {
   u32 chk[8 * K], chv[8 * K];
   u32 warp_tot[32];
   u32 total;
+  u32 done;
 };
 
 template <int K>
@@ -287,14 +296,21 @@ __global__ void __launch_bounds__(ANT + 32, 1)
   const int DC[8] = {0, 0, -1, 1, -1, 1, -1, 1};
   const u64 tcell = (u64)A.tr * A.M + A.tc;
   ull expanded = 0, inserted = 0, pops = 0, pruned = 0, empty = 0;
+  u32 backoff = 128;
   for (u32 it = 0; it < budget; ++it) {
-    const u32 c = q.deletemin(S.popk, S.popv, K);
-    if (c == 0) {
+    const u32 c = q.size_hint() ? q.deletemin(S.popk, S.popv, K) : 0u;
+    if (c == 0) {  // nothing in the heap: done if nothing is in flight either (uniform decision)
       ++empty;
-      if (ld_acq64(state + ST_PENDING) == 0) break;
-      __nanosleep(256);
+      if (tid == 0) S.done = ld_acq64(state + ST_PENDING) == 0;
+      cta_bar<ANT>();
+      const bool done = S.done;
+      cta_bar<ANT>();
+      if (done) break;
+      __nanosleep(backoff);
+      backoff = backoff < 8192 ? backoff * 2 : 8192;
       continue;
     }
+    backoff = 128;
     ++pops;
     u32 nch_total = 0;
     for (int base = 0; base < (int)c; base += ANT) {

@@ -47,7 +47,7 @@ def _astar_case(N, M, rate, seed, K, src=None, dst=None):
     g = synth.grid(N, M, rate, seed)
     src = src or (0, 0)
     dst = dst or (N - 1, M - 1)
-    s = apps.AStarSearch(g, src, dst, K=K, capacity=min(max(1 << 20, 4 * N * M), 1 << 27))
+    s = apps.AStarSearch(g, src, dst, K=K, capacity=min(max(1 << 20, 4 * N * M), 1 << 30))
     s.seed()
     inc, _, _ = apps.run_search(s)
     want = oracle.astar(g, src, dst)["cost"]
