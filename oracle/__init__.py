@@ -71,6 +71,9 @@ def lib():
         L.orc_check_invariants.argtypes = [ctypes.c_uint32, ctypes.c_uint32, ctypes.c_uint32,
                                            ctypes.c_uint32, ctypes.c_uint32, _u32p, _u32p, _u64p]
         L.orc_check_invariants.restype = ctypes.c_int
+        for nm in ("orc_binheap_phased", "orc_sort_phased"):
+            getattr(L, nm).argtypes = [_u32p, ctypes.c_uint64, _u32p]
+            getattr(L, nm).restype = ctypes.c_uint64
         for nm in ("orc_ks_dp", "orc_ks_brute"):
             getattr(L, nm).argtypes = [ctypes.c_uint32, _u32p, _u32p, ctypes.c_uint64]
             getattr(L, nm).restype = ctypes.c_longlong
@@ -136,6 +139,22 @@ def pq_phased(keys, K):
     out = np.empty_like(keys)
     c = lib().orc_pq_phased(_p32(keys), len(keys), K, _p32(out))
     return out[:c]
+
+
+def binheap_phased(keys):
+    """Baseline (not a pin): the phased workload through std::priority_queue, one key per op."""
+    keys = _u32(keys)
+    out = np.empty_like(keys)
+    lib().orc_binheap_phased(_p32(keys), len(keys), _p32(out))
+    return out
+
+
+def sort_phased(keys):
+    """Baseline (not a pin): the closed form of the phased workload, std::sort."""
+    keys = _u32(keys)
+    out = np.empty_like(keys)
+    lib().orc_sort_phased(_p32(keys), len(keys), _p32(out))
+    return out
 
 
 class SeqBGPQ:
