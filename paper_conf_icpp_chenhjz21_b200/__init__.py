@@ -121,7 +121,9 @@ EXPORTS = ("bgpq_create", "bgpq_create_ex", "bgpq_destroy", "bgpq_insert", "bgpq
            "bgpq_size", "bgpq_insert_host", "bgpq_deletemin_host", "bgpq_run_mixed", "bgpq_dump",
            "bgpq_slots", "bgpq_stats", "bgpq_set_grid", "bgpq_grid", "bgpq_launch_count",
            "bgpq_last_error", "bgpq_last_error_msg", "bgpq_strerror", "bgpq_set_debug", "bgpq_timers",
-           "bgpq_test_prim")
+           "bgpq_test_prim", "bgpq_view")
+# every symbol include/bgpq_apps.h declares
+APP_EXPORTS = ("bgpq_ks_prepare", "bgpq_ks_root", "bgpq_ks_run", "bgpq_astar_init", "bgpq_astar_run")
 
 
 class BGPQError(RuntimeError):

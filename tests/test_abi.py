@@ -12,8 +12,8 @@ import paper_conf_icpp_chenhjz21_b200 as pkg
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
-def _declared_functions():
-    src = open(os.path.join(ROOT, "include", "bgpq.h")).read()
+def _declared_functions(header="bgpq.h"):
+    src = open(os.path.join(ROOT, "include", header)).read()
     src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
     return sorted(set(re.findall(r"\b(bgpq_[a-z_]+)\s*\(", src)))
 
@@ -26,6 +26,9 @@ def test_library_builds_and_exports_header_symbols():
     missing = [f for f in declared if not hasattr(L, f)]
     assert not missing, missing
     assert set(declared) == set(pkg.EXPORTS)
+    apps_declared = _declared_functions("bgpq_apps.h")
+    assert set(apps_declared) == set(pkg.APP_EXPORTS)
+    assert not [f for f in apps_declared if not hasattr(L, f)]
 
 
 def test_library_is_sm100a():
