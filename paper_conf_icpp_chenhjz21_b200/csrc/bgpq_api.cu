@@ -58,6 +58,8 @@ struct bgpq {
   u32* stage_v = nullptr;
   u64* stage_cnt = nullptr;
   u64 stage_n = 0;
+  int ds_clusters = -1;    // co-resident clusters of the cluster DELETEMIN engine (-1: not queried)
+  u64* ds_base = nullptr;  // device: ops of the current deletemin call done by that engine
   bool attr_dt = false;    // kernel attributes set / occupancy checked on q->device
   bool attr_pipe = false;
 };
@@ -163,16 +165,53 @@ int ensure_dt(bgpq* q) {
   const size_t n = dt_tasks(q);
   bool ok = cudaMalloc(&D.task_node, n * sizeof(u32)) == cudaSuccess;
   ok = ok && cudaMalloc(&D.task_seq, n * sizeof(u32)) == cudaSuccess;
+  ok = ok && cudaMalloc(&D.task_go, n * sizeof(u64)) == cudaSuccess;
   ok = ok && cudaMalloc(&D.ctl, 32 * sizeof(u32)) == cudaSuccess;
   if (!ok) {
     cudaGetLastError();
     return fail(BGPQ_ENOMEM);
   }
-  if (cudaMemset(D.task_seq, 0, n * sizeof(u32)) != cudaSuccess ||
+  if (cudaMemset(D.task_seq, 0, n * sizeof(u32)) != cudaSuccess || cudaMemset(D.task_go, 0, n * sizeof(u64)) != cudaSuccess ||
       cudaMemset(D.ctl, 0, 32 * sizeof(u32)) != cudaSuccess)
     return fail(BGPQ_ECUDA);
   D.epoch = 0;
+  if (cudaMalloc(&q->ds_base, sizeof(u64)) != cudaSuccess) {
+    cudaGetLastError();
+    return fail(BGPQ_ENOMEM);
+  }
   q->dt_ok = true;
+  return BGPQ_OK;
+}
+
+// The cluster engine (bgpq_dsys.cuh) runs the steady state of a deletemin call first when the
+// output is 16-B aligned for its bulk stores and enough clusters are co-resident (debug bit 256
+// disables it for A/B comparisons).
+bool ds_usable(bgpq* q, const CallArgs& C) {
+  if (g_debug & 256u) return false;
+  if (q->K < 256) return false;
+  if ((reinterpret_cast<uintptr_t>(C.out_k) & 15u) || (C.out_v && (reinterpret_cast<uintptr_t>(C.out_v) & 15u)))
+    return false;
+  if (C.n < (u64)q->K) return false;
+  if (q->ds_clusters < 0) {
+    int cl = 0;
+    if (ktab(q)->ds_prepare(q->sm_count, &cl) != cudaSuccess) {
+      cudaGetLastError();
+      cl = 0;
+    }
+    q->ds_clusters = cl;
+  }
+  return q->ds_clusters >= 8;  // the role cluster + >= 7 clusters of walkers
+}
+
+int dt_epoch(bgpq* q, cudaStream_t s) {
+  DtArgs& D = q->dt;
+  D.epoch += 1;
+  if (D.epoch == 0) {  // wrapped: clear the stale epochs
+    D.epoch = 1;
+    if (cudaMemsetAsync(D.task_seq, 0, dt_tasks(q) * sizeof(u32), s) != cudaSuccess) return fail(BGPQ_ECUDA);
+    if (cudaMemsetAsync(D.task_go, 0, dt_tasks(q) * sizeof(u64), s) != cudaSuccess) return fail(BGPQ_ECUDA);
+  }
+  if (cudaMemsetAsync(D.ctl, 0, 2 * sizeof(u32), s) != cudaSuccess) return fail(BGPQ_ECUDA);
   return BGPQ_OK;
 }
 
@@ -180,13 +219,19 @@ int run_call(bgpq* q, const CallArgs& C, cudaStream_t s) {
   const bool V = (q->flags & BGPQ_FLAG_VALUES) != 0;
   if (C.mode == MODE_DELETEMIN && dt_mode(q)) {
     if (int rc = ensure_dt(q)) return rc;
-    DtArgs& D = q->dt;
-    D.epoch += 1;
-    if (D.epoch == 0) {  // wrapped: clear the stale epochs
-      D.epoch = 1;
-      if (cudaMemsetAsync(D.task_seq, 0, dt_tasks(q) * sizeof(u32), s) != cudaSuccess) return fail(BGPQ_ECUDA);
+    DtArgs D = q->dt;
+    D.op_base = nullptr;
+    if (ds_usable(q, C)) {  // steady state on the cluster engine, the rest on the top CTA
+      if (int rc = dt_epoch(q, s)) return rc;
+      D = q->dt;
+      D.op_base = q->ds_base;
+      if (counted(ktab(q)->ds_launch(q->ds_clusters * DS_CL, heap_args(q), C, D, s)) != cudaSuccess)
+        return fail(BGPQ_ECUDA);
     }
-    if (cudaMemsetAsync(D.ctl, 0, 2 * sizeof(u32), s) != cudaSuccess) return fail(BGPQ_ECUDA);
+    if (int rc = dt_epoch(q, s)) return rc;
+    const u64* base = D.op_base;
+    D = q->dt;
+    D.op_base = const_cast<u64*>(base);
     if (counted(ktab(q)->dt_launch(q->sm_count, heap_args(q), C, D, s)) != cudaSuccess) return fail(BGPQ_ECUDA);
     return BGPQ_OK;
   }
@@ -271,6 +316,8 @@ void bgpq_destroy(bgpq_t* q) {
   cudaFree(q->stage_cnt);
   cudaFree(q->dt.task_node);
   cudaFree(q->dt.task_seq);
+  cudaFree(q->dt.task_go);
+  cudaFree(q->ds_base);
   cudaFree(q->dt.ctl);
   PipeArgs& P = q->pipe;
   u32* pbufs[] = {P.ctl, P.sbk, P.sbv, P.sready, P.rk, P.rv, P.rhdr, P.rflag};

@@ -1,0 +1,905 @@
+// bgpq_dsys.cuh — DELETEMIN calls on a 3-CTA thread-block cluster (B200 design of Alg.2+3 for
+// the steady state of deletemin-only calls; the first stage of bgpq_deletemin).
+//
+// Why.  Alg.3 chains consecutive DELETEMINs: op i+1's depth-0 SORT_SPLIT (l.10) reads the node
+// op i's depth-1 step produced (l.11-15).  On one SM the three SORT_SPLITs of a slot (depth 0
+// and 1 of op i, the lagged depth 2) share the issue and shared-memory bandwidth (~3.3k cycles
+// together, ~0.9-1.5k alone) and one thread's decisions serialise around them (bgpq_dtop.cuh:
+// ~9k cycles per op).  Here every on-chip depth has its own SM: a cluster of three CTAs, a
+// systolic array over the top of the heap, connected by distributed shared memory (DSMEM):
+//   R0 (cluster rank 0): root, nodes 2-3.  Root section of Alg.2 (output of the root, refill
+//       from the last node — taken ahead by R0's helper warp, R20), depth-0 step of Alg.3.
+//   R1 (rank 1): nodes 4-7.  Depth-1 step (SORT_SPLIT of y1's children, l.10; (y1, y2) split,
+//       l.12); the new y1 is pushed into R0's shared memory by a DSMEM bulk copy.
+//   R2 (rank 2): nodes 8-15.  Depth-2 step, pushes y2 to R1; hands y3 (LOCKed) with the
+//       carried keys to a walker CTA (blockIdx >= 3: dt_walk, Alg.3 from l.2 with the paper's
+//       hand-over-hand locks) and, through its helper warp, re-loads y3 once the walker has
+//       released it (the node is "lent" meanwhile).
+// Every level runs op i's step only after the level above sent op i's path node y_d (message
+// "a", sent as soon as it is known from the children's cached max keys, l.9 — before the
+// level's own SORT_SPLIT) and commits it after message "b" (the carried keys' descriptor and
+// whether the walk continues, l.4).  Each level applies the ops in call order, so every node
+// sees exactly the sequence of steps of the sequential execution of Alg.2+3 in call order,
+// except for the early refill take (R20): linearizable with linearization order = call order.
+// Carried keys (the refill node's keys as they sink, l.12 swaps in >99% of top-level steps)
+// travel by reference: a global node index whose HBM copy holds them (the refill node, EMPTY
+// after the take and never written during the call) — materialised only when a (cur, y)
+// SORT_SPLIT really merges (then into the HBM copy of the on-chip node y_d, dead while on chip).
+//
+// Scope: full-K DELETEMINs while heapSize >= DS_HMIN, |root| = K, empty pBuffer (the state of
+// a drain after insert calls of whole batches).  The rest of the call (partial batches, small
+// heaps, non-empty buffers) is executed by bgpq_dtop_kernel, launched right after on the same
+// stream, which reads how many ops this kernel did (DtArgs::op_base).
+#pragma once
+#include "bgpq_dtop.cuh"
+
+namespace bgpqd {
+
+constexpr int DS_NT = 512;             // compute threads per CTA
+constexpr int DS_BLOCK = DS_NT + 64;   // + 2 helper warps (roles) / lock warp + idle warp (walkers)
+constexpr int DS_CL = 5;               // cluster size: steps of depths 0 .. DS_CL-1 in the cluster
+constexpr int DS_NSLOT = 24;           // node slots per role CTA
+constexpr u32 DS_MAXOWN = 1u << (DS_CL - 1);  // nodes the deepest owning level holds (depth DS_CL-1)
+constexpr u32 DS_RING = 16;            // inbox entries
+constexpr u32 DS_CREDIT = 4;           // credits are returned every DS_CREDIT entries
+constexpr u32 DS_RF = 8;               // refill takes run at most this many ops ahead (R20)
+constexpr u32 DS_HMIN = 1024;          // heapSize floor of the engine (depth >= 10 > DS_RF)
+constexpr u32 DS_NONE = 0xFFFFFFFFu;
+
+enum : u32 { MK_A = 1, MK_ASTOP = 2, MK_B = 3, MK_BSTOP = 4 };
+
+
+struct __align__(16) DsMsg {
+  u32 op, kind, y, slot, src, cmin, cmax, pad;
+};
+
+// per role CTA control block (same layout in every CTA of the cluster: DSMEM addresses are
+// obtained with mapa from local addresses)
+struct DsCtl {
+  u64 inbar[DS_RING];    // inbox entry barriers: armed (expect_tx) by this CTA, completed by the
+                         // sender's bulk copy of the message (async proxy: no sender-side fence)
+  u64 slotbar[DS_NSLOT]; // push completion per slot: armed by this CTA when it designates the slot
+  DsMsg stage[DS_RING];  // outgoing messages (source of the bulk copies)
+  u64 ainbar[DS_RING];   // second inbox (path messages "a" for the stager's staging helper)
+  DsMsg ainbox[DS_RING];
+  DsMsg astage[DS_RING];
+  u32 aconsumed;
+  u64 lbar;              // local TMA loads
+  u64 hbar;              // helper's TMA loads
+  u64 sbar[4];           // stager: staging completion of the op in staging ring entry k % 4
+  DsMsg inbox[DS_RING];
+  u32 consumed;          // inbox entries consumed (written remotely by the receiver into the SENDER,
+                         // every DS_CREDIT entries)
+  u32 b[16];             // thread-0 broadcasts
+  // R0 helper: refill takes
+  u32 rf_seq;            // takes published
+  u32 rf_min[DS_RF], rf_max[DS_RF];
+  u32 rf_used;           // ops whose take thread 0 consumed
+  // stager: helper A (LOCK + stage children) and helper B (tasks, write-backs, UNLOCKs) rings
+  u32 sq_done;           // staging records published (helper A -> thread 0), one per op
+  u32 sq_ret;            // ops whose staging slots thread 0 returned
+  u32 stg_y[16], stg_up[16], stg_min[16][2], stg_max[16][2];
+  u32 wq_head, wq_done, wq[16 * 5];
+  u32 wb_free;           // slots helper B finished reading (atomicOr; thread 0 collects)
+  u32 tasks;             // walker tasks published
+  u32 quit;
+  // thread-0 node table (shared memory, not local arrays: cluster-scope acquires invalidate
+  // L1, so local memory would cost an L2 round trip per access)
+  u32 ns[DS_MAXOWN], mn[DS_MAXOWN], mx[DS_MAXOWN], pend[DS_MAXOWN];
+  ull st[NSTAT];
+  ull tm[8];  // debug timers (bgpq_set_debug bit 1024): total, wait-above, wait-children, split, wait-b, sends
+};
+constexpr size_t DSCTL_BYTES = (sizeof(DsCtl) + 127) / 128 * 128;
+
+template <int K, bool V>
+constexpr size_t ds_smem_bytes() {
+  const size_t role = DSCTL_BYTES + (size_t)DS_NSLOT * K * 4 * (V ? 2 : 1);
+  const size_t wrk = LCTL_BYTES + (size_t)LSLOT * K * 4 * (V ? 2 : 1);
+  return role > wrk ? role : wrk;
+}
+
+// ---- cluster / DSMEM PTX -----------------------------------------------------------------
+__device__ __forceinline__ u32 cl_rank() {
+  u32 r;
+  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+  return r;
+}
+__device__ __forceinline__ u32 cl_map(const void* p, u32 rank) {  // local smem -> cluster address in `rank`
+  u32 a;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(a) : "r"(smem_addr(p)), "r"(rank));
+  return a;
+}
+__device__ __forceinline__ void cl_st(u32 addr, u32 v) {
+  asm volatile("st.shared::cluster.u32 [%0], %1;" ::"r"(addr), "r"(v) : "memory");
+}
+__device__ __forceinline__ void cl_st_release(u32 addr, u32 v) {
+  asm volatile("st.release.cluster.shared::cluster.u32 [%0], %1;" ::"r"(addr), "r"(v) : "memory");
+}
+__device__ __forceinline__ u32 ld_acq_cluster(const u32* p) {
+  u32 v;
+  asm volatile("ld.acquire.cluster.shared::cta.u32 %0, [%1];" : "=r"(v) : "r"(smem_addr(p)) : "memory");
+  return v;
+}
+__device__ __forceinline__ void cl_arrive(u32 bar_addr) {
+  asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(bar_addr) : "memory");
+}
+__device__ __forceinline__ void cl_arrive_tx(u32 bar_addr, u32 bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.release.cluster.shared::cluster.b64 _, [%0], %1;" ::"r"(bar_addr),
+               "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait_cluster(u64* bar, u32 phase) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n"
+      "WAITC_%=:\n\t"
+      "mbarrier.try_wait.parity.acquire.cluster.shared::cta.b64 p, [%0], %1;\n\t"
+      "@!p bra WAITC_%=;\n}" ::"r"(smem_addr(bar)),
+      "r"(phase) : "memory");
+}
+// bulk copy of `bytes` from this CTA's smem to a cluster address, completing tx on a
+// (remote) mbarrier
+__device__ __forceinline__ void bulk_s2cl(u32 dst, const void* src, u32 bytes, u32 bar) {
+  asm volatile("cp.async.bulk.shared::cluster.shared::cta.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
+               "r"(smem_addr(src)), "r"(bytes), "r"(bar) : "memory");
+}
+__device__ __forceinline__ void cluster_sync_all() {
+  asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+
+// =========================================================================================
+// One role CTA of the cluster
+// =========================================================================================
+template <int K, bool V>
+struct DsRole {
+  static constexpr u32 NB = K * 4u;
+  static constexpr u32 SLOTB = V ? 2u * NB : NB;
+  HeapArgs H;
+  CallArgs C;
+  DtArgs D;
+  DsCtl* c;
+  u32* sk;
+  u32* sv;
+  u32 rank;
+  // thread-0 state (registers)
+  u32 fm;                 // free slot mask
+  u32 sbph;               // slot barrier parities (bit s)
+  u32 in_seq;             // inbox entries consumed
+  u32 out_seq;            // messages sent to the level below
+  u32 out_seq2;           // path messages sent to the stager's second inbox
+  u32 lph;                // lbar parity
+  bool timing;
+  __device__ __forceinline__ ull tnow() const { return timing ? clock64() : 0ull; }
+  __device__ __forceinline__ void tacc(int k, ull t0) { if (timing) c->tm[k] += clock64() - t0; }
+
+  __device__ __forceinline__ u32* BK(u32 s) const { return sk + s * K; }
+  __device__ __forceinline__ u32* BV(u32 s) const { return V ? sv + s * K : nullptr; }
+  __device__ __forceinline__ u32 alloc() {
+    if (fm == 0) __trap();
+    const u32 s = __ffs(fm) - 1;
+    fm &= ~(1u << s);
+    return s;
+  }
+  __device__ __forceinline__ void release(u32 s) {
+    if (s != DS_NONE) fm |= 1u << s;
+  }
+  // ---- inbox (thread 0).  A message is a 32-B bulk copy from the sender's staging ring into
+  // this CTA's inbox entry, completing the entry's barrier (armed here with expect_tx); so the
+  // sender needs no cluster-scope release and the receiver waits at CTA scope.
+  __device__ __forceinline__ void arm_inbox(u32 e) {
+    mbar_arrive_expect_tx(&c->inbar[e], (u32)sizeof(DsMsg));
+  }
+  __device__ __forceinline__ DsMsg recv() {
+    const u32 e = in_seq % DS_RING;
+    mbar_wait(&c->inbar[e], (in_seq / DS_RING) & 1u);
+    DsMsg m;
+    volatile DsMsg* pm = &c->inbox[e];
+    m.op = pm->op; m.kind = pm->kind; m.y = pm->y; m.slot = pm->slot;
+    m.src = pm->src; m.cmin = pm->cmin; m.cmax = pm->cmax;
+    ++in_seq;
+    arm_inbox(e);  // for the message DS_RING entries later
+    if (in_seq % DS_CREDIT == 0) {  // credit back to the sender (its staging entries are free too)
+      const ull t0 = tnow();
+      asm volatile("st.relaxed.cluster.shared::cluster.u32 [%0], %1;" ::"r"(cl_map(&c->consumed, rank - 1)),
+                   "r"(in_seq) : "memory");
+      tacc(6, t0);
+    }
+    return m;
+  }
+  // ---- send to the level below (thread 0)
+  __device__ __forceinline__ void send(u32 op, u32 kind, u32 y = 0, u32 slot = 0, u32 src = 0, u32 cmin = 0,
+                                       u32 cmax = 0) {
+    const ull t0 = tnow();
+    while (out_seq - *reinterpret_cast<volatile u32*>(&c->consumed) >= DS_RING - DS_CREDIT) {}
+    const u32 e = out_seq % DS_RING;
+    const u32 dst = rank + 1;
+    DsMsg& m = c->stage[e];
+    m.op = op; m.kind = kind; m.y = y; m.slot = slot; m.src = src; m.cmin = cmin; m.cmax = cmax; m.pad = 0;
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    bulk_s2cl(cl_map(&c->inbox[e], dst), &m, (u32)sizeof(DsMsg), cl_map(&c->inbar[e], dst));
+    asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+    ++out_seq;
+    tacc(5, t0);
+  }
+  // ---- path messages to the stager go to its second inbox (read by its staging helper)
+  __device__ __forceinline__ void send_a2(u32 op, u32 kind, u32 y, u32 slot) {
+    const ull t0 = tnow();
+    while (out_seq2 - *reinterpret_cast<volatile u32*>(&c->aconsumed) >= DS_RING - DS_CREDIT) {}
+    const u32 e = out_seq2 % DS_RING;
+    const u32 dst = rank + 1;
+    DsMsg& m = c->astage[e];
+    m.op = op; m.kind = kind; m.y = y; m.slot = slot; m.src = 0; m.cmin = 0; m.cmax = 0; m.pad = 0;
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    bulk_s2cl(cl_map(&c->ainbox[e], dst), &m, (u32)sizeof(DsMsg), cl_map(&c->ainbar[e], dst));
+    asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+    ++out_seq2;
+    tacc(5, t0);
+  }
+  __device__ __forceinline__ void send_path(u32 op, u32 kind, u32 y = 0, u32 slot = 0) {
+    if (rank + 2 == (u32)DS_CL) send_a2(op, kind, y, slot);
+    else send(op, kind, y, slot);
+  }
+  // ---- slots the level below pushes into: armed when designated, disarmed if no push comes
+  __device__ __forceinline__ void arm_slot(u32 s) { mbar_arrive_expect_tx(&c->slotbar[s], SLOTB); }
+  __device__ __forceinline__ void disarm_slot(u32 s) {
+    asm volatile("mbarrier.complete_tx.relaxed.cta.shared::cta.b64 [%0], %1;" ::"r"(smem_addr(&c->slotbar[s])),
+                 "r"(SLOTB) : "memory");
+    wait_pushed(s);
+  }
+  // ---- push slot s (K entries) into slot `ds` of the level above, which armed it (thread 0;
+  // the caller made the slot's generic writes visible with a CTA barrier)
+  __device__ __forceinline__ void push_up(u32 s, u32 ds) {
+    const ull t0 = tnow();
+    const u32 up = rank - 1;
+    const u32 bar = cl_map(&c->slotbar[ds], up);
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    bulk_s2cl(cl_map(BK(ds), up), BK(s), NB, bar);
+    if (V) bulk_s2cl(cl_map(BV(ds), up), BV(s), NB, bar);
+    asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+    tacc(7, t0);
+  }
+  __device__ __forceinline__ void wait_pushed(u32 s) {  // a push into local slot s has landed
+    mbar_wait(&c->slotbar[s], (sbph >> s) & 1u);
+    sbph ^= 1u << s;
+  }
+  // synchronous TMA load of HBM node n into slot s (thread 0)
+  __device__ __forceinline__ void load_node(u32 s, u32 n) {
+    fence_proxy_async();
+    mbar_arrive_expect_tx(&c->lbar, SLOTB);
+    bulk_g2s(BK(s), H.gk + (size_t)n * K, NB, &c->lbar);
+    if (V) bulk_g2s(BV(s), H.gv + (size_t)n * K, NB, &c->lbar);
+    mbar_wait(&c->lbar, lph);
+    lph ^= 1u;
+  }
+  // write slot s to HBM node n (thread 0, TMA bulk store, waits for completion)
+  __device__ __forceinline__ void store_node(u32 n, u32 s) {
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    bulk_s2g(H.gk + (size_t)n * K, BK(s), NB);
+    if (V) bulk_s2g(H.gv + (size_t)n * K, BV(s), NB);
+    asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+    asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+  }
+};
+
+// All NT compute threads: SORT_SPLIT of two full K-batches, X = K smallest, Y = rest.
+template <int K, bool V>
+__device__ __forceinline__ void ds_split(DsRole<K, V>& R, u32 z, u32 w, u32 x, u32 y) {
+  cta_bar<DS_NT>();
+  sort_split<K, DS_NT, V>(R.BK(z), R.BV(z), K, R.BK(w), R.BV(w), K, K, R.BK(x), R.BV(x), R.BK(y), R.BV(y));
+  cta_bar<DS_NT>();
+}
+
+// Number of full-K ops the engine executes (identical in every role CTA): the call's full
+// batches, while heapSize stays >= DS_HMIN, if |root| = K and the pBuffer is empty.
+__device__ __forceinline__ u64 ds_ops(const HeapArgs& H, const CallArgs& C, int K) {
+  const u32 hs = ld_relaxed(H.hdr + H_HS), rs = ld_relaxed(H.hdr + H_RS), ps = ld_relaxed(H.hdr + H_PS);
+  if (rs != (u32)K || ps != 0 || hs < DS_HMIN + 2) return 0;
+  const u64 full = C.n / (u64)K;
+  const u64 room = hs - DS_HMIN;
+  return full < room ? full : room;
+}
+
+// -----------------------------------------------------------------------------------------
+// R0: root section + depth 0
+// -----------------------------------------------------------------------------------------
+template <int K, bool V>
+__device__ void ds_r0(DsRole<K, V>& R, const u64 m) {
+  DsCtl* c = R.c;
+  const HeapArgs& H = R.H;
+  const int tid = threadIdx.x;
+  u32 hs = ld_relaxed(H.hdr + H_HS);
+  // on-chip nodes: 1 (root), 2, 3
+  u32* ns = c->ns;
+  u32* mn = c->mn;
+  u32* mx = c->mx;
+  u32* pend = c->pend;
+  if (tid == 0) {
+    for (u32 q = 1; q <= 3; ++q) {
+      ns[q] = R.alloc();
+      pend[q] = 0;
+      mn[q] = ld_relaxed(&H.meta[q].kmin);
+      mx[q] = ld_relaxed(&H.meta[q].kmax);
+    }
+    fence_proxy_async();
+    mbar_arrive_expect_tx(&c->lbar, 3u * DsRole<K, V>::SLOTB);
+    for (u32 q = 1; q <= 3; ++q) {
+      bulk_g2s(R.BK(ns[q]), H.gk + (size_t)q * K, DsRole<K, V>::NB, &c->lbar);
+      if (V) bulk_g2s(R.BV(ns[q]), H.gv + (size_t)q * K, DsRole<K, V>::NB, &c->lbar);
+    }
+    mbar_wait(&c->lbar, R.lph);
+    R.lph ^= 1u;
+  }
+  cta_bar<DS_NT>();
+  u32 out_old = DS_NONE;  // root slot whose output store may still be reading it
+  const ull t_start = R.tnow();
+  for (u64 i = 0; i < m; ++i) {
+    if (tid == 0) {
+      // refill of op i (Alg.2 l.5-12), taken ahead by the helper: node hs, now EMPTY
+      const u32 t = hs;
+      const ull t1 = R.tnow();
+      while (ld_acq_cta(&c->rf_seq) <= (u32)i) {}
+      R.tacc(1, t1);
+      const u32 rmin = c->rf_min[i % DS_RF], rmax = c->rf_max[i % DS_RF];
+      st_rel_cta(&c->rf_used, (u32)i + 1u);
+      hs -= 1;
+      // a pending y1 push of op i-1 must have landed before depth 0 reads it
+      const ull t2 = R.tnow();
+      for (u32 q = 2; q <= 3; ++q)
+        if (pend[q]) {
+          R.wait_pushed(ns[q]);
+          pend[q] = 0;
+          mn[q] = R.BK(ns[q])[0];
+          mx[q] = R.BK(ns[q])[K - 1];
+        }
+      R.tacc(2, t2);
+      // Alg.2 l.22: the root's K keys are op i's output (TMA bulk store, async)
+      asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");  // the previous output's read
+      R.release(out_old);
+      const u64 pos = i * (u64)K;
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      bulk_s2g(R.C.out_k + pos, R.BK(ns[1]), DsRole<K, V>::NB);
+      if (V && R.C.out_v) bulk_s2g(R.C.out_v + pos, R.BV(ns[1]), DsRole<K, V>::NB);
+      asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+      out_old = ns[1];
+      c->st[S_DEL_OPS]++;
+      c->st[S_DEL_REFILL]++;
+      // Alg.3 at the root: cur = root holding the refill keys (R3: |root| = K = size refills)
+      const u32 minc = mn[2] < mn[3] ? mn[2] : mn[3];
+      if (rmax <= minc) {  // l.4: stop at the root — root <- the refill keys
+        const u32 s = R.alloc();
+        R.load_node(s, t);
+        ns[1] = s; mn[1] = rmin; mx[1] = rmax;
+        R.send((u32)i, MK_ASTOP);
+        c->b[0] = 1;
+      } else {
+        const u32 x = mx[2] > mx[3] ? 2u : 3u, y = 5u - x;  // l.9 (R6: tie -> x = r)
+        const u32 sy = R.alloc();  // y1's new content arrives here from R1
+        R.arm_slot(sy);
+        R.send((u32)i, MK_A, y, sy);
+        const u32 A = R.alloc(), B = R.alloc();
+        c->b[0] = 0; c->b[1] = ns[2]; c->b[2] = ns[3]; c->b[3] = A; c->b[4] = B;
+        c->b[5] = x; c->b[6] = y; c->b[7] = sy; c->b[8] = t; c->b[9] = rmin; c->b[10] = rmax;
+        c->st[S_DEL_LEVELS]++;
+        c->st[(mx[2] <= mn[3] || mx[3] <= mn[2]) ? S_DEL_LR_NOMOVE : S_DEL_LR_MERGE]++;
+      }
+    }
+    cta_bar<DS_NT>();
+    if (c->b[0]) continue;
+    const u32 s2 = c->b[1], s3 = c->b[2], A = c->b[3], B = c->b[4];
+    const ull t3 = R.tnow();
+    ds_split<K, V>(R, s2, s3, A, B);  // l.10: (Heap[y], Heap[x]) <- SORT_SPLIT(l, r)
+    if (tid == 0) R.tacc(3, t3);
+    if (tid == 0) {
+      const u32 x = c->b[5], y = c->b[6], sy = c->b[7], t = c->b[8], rmin = c->b[9], rmax = c->b[10];
+      R.release(s2); R.release(s3);
+      const u32 ymax = R.BK(A)[K - 1];
+      if (ymax <= rmin) {  // l.12 is a swap: root <- Y, the refill keys sink on (by reference)
+        ns[1] = A; mn[1] = R.BK(A)[0]; mx[1] = ymax;
+        c->st[S_DEL_CY_SWAP]++;
+        R.send((u32)i, MK_B, 0, 0, t, rmin, rmax);
+      } else {  // l.12 merges: (root, C1) <- SORT_SPLIT(refill, Y); C1 into y1's dead HBM copy
+        const u32 r = R.alloc(), lo = R.alloc(), hi = R.alloc();
+        R.load_node(r, t);
+        c->b[11] = r; c->b[12] = lo; c->b[13] = hi; c->b[14] = 1;
+      }
+      ns[x] = B; mn[x] = R.BK(B)[0]; mx[x] = R.BK(B)[K - 1];
+      ns[y] = sy; pend[y] = 1;
+      if (!(ymax <= rmin)) c->b[15] = 1; else c->b[15] = 0;
+    }
+    cta_bar<DS_NT>();
+    if (c->b[15]) {  // rare: a real (cur, y) merge at the root
+      const u32 r = c->b[11], lo = c->b[12], hi = c->b[13];
+      ds_split<K, V>(R, r, A, lo, hi);
+      if (tid == 0) {
+        const u32 y = c->b[6];
+        R.store_node(y, hi);  // C1 in y1's HBM copy (y1 is on chip; its HBM copy is dead)
+        __threadfence();
+        R.send((u32)i, MK_B, 0, 0, y, R.BK(hi)[0], R.BK(hi)[K - 1]);
+        ns[1] = lo; mn[1] = R.BK(lo)[0]; mx[1] = R.BK(lo)[K - 1];
+        R.release(r); R.release(hi); R.release(A);
+      }
+      cta_bar<DS_NT>();
+    }
+  }
+  // ---- end: wait for the last pushes, write the on-chip nodes back, update the header
+  if (tid == 0) {
+    R.tacc(0, t_start);
+    for (u32 q = 2; q <= 3; ++q)
+      if (pend[q]) { R.wait_pushed(ns[q]); pend[q] = 0; mn[q] = R.BK(ns[q])[0]; mx[q] = R.BK(ns[q])[K - 1]; }
+    asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+    for (u32 q = 1; q <= 3; ++q) {
+      R.store_node(q, ns[q]);
+      st_relaxed(&H.meta[q].kmin, mn[q]);
+      st_relaxed(&H.meta[q].kmax, mx[q]);
+    }
+    st_relaxed(H.hdr + H_HS, hs);
+    ull lin;
+    asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(lin) : "l"(H.hdr + H_LIN) : "memory");
+    asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(H.hdr + H_LIN), "l"(lin + m) : "memory");
+    c->st[S_KEYS_OUT] += m * (u64)K;
+    if (R.C.d_count && m) atomicAdd(R.C.d_count, (ull)(m * (u64)K));
+    *reinterpret_cast<volatile u64*>(R.D.op_base) = m;
+    c->quit = 1;
+  }
+}
+
+// R0's helper (lane 0): the refill takes (Alg.2 l.6-12) up to DS_RF ops ahead (R20).
+template <int K, bool V>
+__device__ void ds_r0_helper(DsRole<K, V>& R, const u64 m) {
+  DsCtl* c = R.c;
+  const HeapArgs& H = R.H;
+  const u32 hs0 = ld_relaxed(H.hdr + H_HS);
+  for (u64 j = 0; j < m; ++j) {
+    while ((u32)j >= ld_acq_cta(&c->rf_used) + DS_RF) __nanosleep(32);
+    const u32 t = hs0 - (u32)j;
+    lock_acquire(&H.meta[t].lock);  // l.6: LOCK(tar)
+    const u32 mnv = ld_relaxed(&H.meta[t].kmin), mxv = ld_relaxed(&H.meta[t].kmax);
+    st_relaxed(&H.meta[t].state, ST_EMPTY);  // l.11: its keys move to the root, tar <- EMPTY
+    lock_release(&H.meta[t].lock);           // l.12: UNLOCK(tar)
+    // the keys sink by reference (the HBM copy of t): warm them in L2 for the walker that
+    // will load them below the cluster's levels
+    if (!(R.C.debug & 2048u))
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(H.gk + (size_t)t * K), "r"(DsRole<K, V>::NB)
+                 : "memory");
+    if (V && !(R.C.debug & 2048u))
+      asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(H.gv + (size_t)t * K), "r"(DsRole<K, V>::NB)
+                   : "memory");
+    c->rf_min[j % DS_RF] = mnv;
+    c->rf_max[j % DS_RF] = mxv;
+    st_rel_cta(&c->rf_seq, (u32)j + 1u);
+  }
+}
+
+// -----------------------------------------------------------------------------------------
+// R1 .. R(DS_CL-2): the depth-d step (d = rank), owning the nodes of depth d+1
+// -----------------------------------------------------------------------------------------
+template <int K, bool V>
+__device__ void ds_level(DsRole<K, V>& R, const u64 m) {
+  DsCtl* c = R.c;
+  const HeapArgs& H = R.H;
+  const int tid = threadIdx.x;
+  const u32 d = R.rank;              // this CTA's step depth
+  const u32 base = 1u << (d + 1);    // first owned node
+  const u32 cnt = base;              // owned nodes: base .. 2*base-1
+  u32* ns = c->ns;
+  u32* mn = c->mn;
+  u32* mx = c->mx;
+  u32* pend = c->pend;
+  if (tid == 0) {
+    fence_proxy_async();
+    mbar_arrive_expect_tx(&c->lbar, cnt * DsRole<K, V>::SLOTB);
+    for (u32 j = 0; j < cnt; ++j) {
+      const u32 n = base + j;
+      ns[j] = R.alloc();
+      pend[j] = 0;
+      mn[j] = ld_relaxed(&H.meta[n].kmin);
+      mx[j] = ld_relaxed(&H.meta[n].kmax);
+      bulk_g2s(R.BK(ns[j]), H.gk + (size_t)n * K, DsRole<K, V>::NB, &c->lbar);
+      if (V) bulk_g2s(R.BV(ns[j]), H.gv + (size_t)n * K, DsRole<K, V>::NB, &c->lbar);
+    }
+    mbar_wait(&c->lbar, R.lph);
+    R.lph ^= 1u;
+  }
+  cta_bar<DS_NT>();
+  u32 push_old = DS_NONE;  // slot whose push may still be reading it
+  const ull t_start = R.tnow();
+  for (u64 i = 0; i < m; ++i) {
+    if (tid == 0) {
+      const ull t1 = R.tnow();
+      const DsMsg a = R.recv();
+      R.tacc(1, t1);
+      c->b[0] = 0;
+      if (a.kind == MK_ASTOP) {  // the walk stopped above: nothing at this depth
+        R.send_path((u32)i, MK_ASTOP);
+        c->b[0] = 1;
+      } else {
+        const u32 l = 2u * a.y, r = l + 1u, jl = l - base, jr = r - base;
+        const ull t2 = R.tnow();
+        for (u32 q = 0; q < 2; ++q) {  // both children current (their pushes landed)
+          const u32 j = q ? jr : jl;
+          if (pend[j]) {
+            R.wait_pushed(ns[j]);
+            pend[j] = 0;
+            mn[j] = R.BK(ns[j])[0];
+            mx[j] = R.BK(ns[j])[K - 1];
+          }
+        }
+        R.tacc(2, t2);
+        const u32 x = mx[jl] > mx[jr] ? l : r, y = l + r - x;  // l.9 (R6)
+        const u32 sy = R.alloc();  // y's new content arrives here from the level below
+        R.arm_slot(sy);
+        R.send_path((u32)i, MK_A, y, sy);
+        const u32 A = R.alloc(), B = R.alloc();
+        c->b[1] = ns[jl]; c->b[2] = ns[jr]; c->b[3] = A; c->b[4] = B; c->b[5] = x; c->b[6] = y;
+        c->b[7] = sy; c->b[9] = a.slot;
+        c->b[10] = (mx[jl] <= mn[jr] || mx[jr] <= mn[jl]) ? 1u : 0u;
+        c->b[13] = mn[jl] < mn[jr] ? mn[jl] : mn[jr];
+      }
+    }
+    cta_bar<DS_NT>();
+    if (c->b[0]) continue;
+    const u32 sl = c->b[1], sr = c->b[2], A = c->b[3], B = c->b[4];
+    const ull t3 = R.tnow();
+    ds_split<K, V>(R, sl, sr, A, B);  // l.10 (speculative until message b)
+    if (tid == 0) {
+      R.tacc(3, t3);
+      const u32 x = c->b[5], y = c->b[6], sy = c->b[7], up = c->b[9];
+      const u32 minc = c->b[13];
+      const ull t4 = R.tnow();
+      const DsMsg b = R.recv();  // the carried keys of cur (l.12) from the level above
+      R.tacc(4, t4);
+      asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");  // the previous push's read
+      R.release(push_old);
+      push_old = DS_NONE;
+      c->b[14] = 0;
+      if (b.kind == MK_BSTOP) {  // the walk stopped above after all: drop the speculative split
+        R.release(A); R.release(B);
+        R.disarm_slot(sy);
+        R.release(sy);
+        R.send((u32)i, MK_BSTOP);
+      } else if (b.cmax <= minc) {  // l.4: stop at cur — cur keeps the carried keys
+        const u32 s = R.alloc();
+        R.load_node(s, b.src);
+        R.push_up(s, up);
+        push_old = s;
+        R.release(A); R.release(B);
+        R.disarm_slot(sy);
+        R.release(sy);
+        R.send((u32)i, MK_BSTOP);
+      } else {
+        c->st[S_DEL_LEVELS]++;
+        c->st[c->b[10] ? S_DEL_LR_NOMOVE : S_DEL_LR_MERGE]++;
+        const u32 ymax = R.BK(A)[K - 1];
+        const u32 jx = x - base, jy = y - base;
+        R.release(sl); R.release(sr);
+        ns[jx] = B; mn[jx] = R.BK(B)[0]; mx[jx] = R.BK(B)[K - 1];
+        ns[jy] = sy; pend[jy] = 1;
+        if (ymax <= b.cmin) {  // l.12 swap: cur <- Y (pushed up), the carried keys sink on
+          c->st[S_DEL_CY_SWAP]++;
+          R.push_up(A, up);
+          push_old = A;
+          R.send((u32)i, MK_B, 0, 0, b.src, b.cmin, b.cmax);
+        } else {  // l.12 merges: (cur, C) <- SORT_SPLIT(carried, Y); C into y's dead HBM copy
+          const u32 cs = R.alloc(), lo = R.alloc(), hi = R.alloc();
+          R.load_node(cs, b.src);
+          c->b[14] = 1; c->b[4] = cs; c->b[5] = lo; c->b[6] = hi; c->b[7] = y; c->b[9] = up; c->b[12] = A;
+        }
+      }
+    }
+    cta_bar<DS_NT>();
+    if (c->b[14]) {  // rare: a real (cur, y) merge at this depth
+      const u32 cs = c->b[4], lo = c->b[5], hi = c->b[6], Y = c->b[12];
+      ds_split<K, V>(R, cs, Y, lo, hi);
+      if (tid == 0) {
+        const u32 y = c->b[7], up = c->b[9];
+        R.store_node(y, hi);  // the new carried keys in y's HBM copy
+        __threadfence();
+        R.push_up(lo, up);
+        push_old = lo;
+        R.release(cs); R.release(Y);
+        R.send((u32)i, MK_B, 0, 0, y, R.BK(hi)[0], R.BK(hi)[K - 1]);
+        R.release(hi);
+      }
+      cta_bar<DS_NT>();
+    }
+  }
+  // ---- end: pending pushes landed, write the owned nodes back
+  if (tid == 0) {
+    R.tacc(0, t_start);
+    asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+    for (u32 j = 0; j < cnt; ++j) {
+      const u32 n = base + j;
+      if (pend[j]) {
+        R.wait_pushed(ns[j]);
+        pend[j] = 0;
+        mn[j] = R.BK(ns[j])[0];
+        mx[j] = R.BK(ns[j])[K - 1];
+      }
+      R.store_node(n, ns[j]);
+      st_relaxed(&H.meta[n].kmin, mn[j]);
+      st_relaxed(&H.meta[n].kmax, mx[j]);
+    }
+  }
+}
+
+// -----------------------------------------------------------------------------------------
+// R(DS_CL-1), the stager: the depth-(DS_CL-1) step on children staged from HBM (LOCKed by its
+// helper warp A as soon as the level above names the path node), write-back of x and
+// UNLOCK by helper warp B, hand-over of y (still LOCKed) with the carried keys to a walker
+// (published early so the walker LOCKs and stages y's children meanwhile).  Owns no nodes:
+// the new content of its cur is pushed into the level above.
+// -----------------------------------------------------------------------------------------
+enum : u32 { WQ_PUBLISH = 1, WQ_COMMIT = 2, WQ_CANCEL = 3, WQ_WB = 4, WQ_UNLOCK = 5, WQ_END = 6 };
+
+template <int K, bool V>
+__device__ __forceinline__ void sq_req(DsRole<K, V>& R, u32* head, const u32* done, u32* ring, u32 a0, u32 a1,
+                                       u32 a2, u32 a3, u32 a4) {
+  const u32 h = *head;
+  while (h - ld_acq_cta(done) >= 16u) {}
+  u32* e = ring + (h % 16) * 5;
+  e[0] = a0; e[1] = a1; e[2] = a2; e[3] = a3; e[4] = a4;
+  st_rel_cta(head, h + 1u);
+}
+
+template <int K, bool V>
+__device__ void ds_stager(DsRole<K, V>& R, const u64 m) {
+  DsCtl* c = R.c;
+  const int tid = threadIdx.x;
+  u32 sbp = 0;  // parities of sbar[0..3]
+  u32 push_old = DS_NONE;
+  const ull t_start = R.tnow();
+  for (u64 i = 0; i < m; ++i) {
+    if (tid == 0) {
+      const ull t2 = R.tnow();
+      while (ld_acq_cta(&c->sq_done) <= (u32)i) {}  // op i's children LOCKed and staged (helper A)
+      R.tacc(2, t2);
+      c->b[0] = 0;
+      const u32 e = (u32)i % 16;
+      const u32 y4 = c->stg_y[e];
+      if (y4 == 0) {  // the walk stopped above
+        c->b[0] = 1;
+        st_rel_cta(&c->sq_ret, (u32)i + 1u);
+      } else {
+        const u32 l = 2u * y4, r = l + 1u;
+        const u32 sl = DS_NSLOT - 8 + 2 * (u32)(i % 4), sr = sl + 1;
+        mbar_wait(&c->sbar[i % 4], sbp >> (i % 4) & 1u);  // the staged data
+        sbp ^= 1u << (i % 4);
+        const u32 lmin = c->stg_min[e][0], lmax = c->stg_max[e][0], rmin = c->stg_min[e][1], rmax = c->stg_max[e][1];
+        const u32 x = lmax > rmax ? l : r, y = l + r - x;  // l.9 (R6)
+        sq_req<K, V>(R, &c->wq_head, &c->wq_done, c->wq, WQ_PUBLISH, y, 0, 0, 0);
+        const u32 A = R.alloc(), B = R.alloc();
+        c->b[1] = sl; c->b[2] = sr; c->b[3] = A; c->b[4] = B; c->b[5] = x; c->b[6] = y; c->b[9] = c->stg_up[e];
+        c->b[10] = (lmax <= rmin || rmax <= lmin) ? 1u : 0u;
+        c->b[13] = lmin < rmin ? lmin : rmin;
+        c->b[11] = l; c->b[12] = r;
+      }
+    }
+    cta_bar<DS_NT>();
+    if (c->b[0]) continue;
+    const u32 sl = c->b[1], sr = c->b[2], A = c->b[3], B = c->b[4];
+    const ull t3 = R.tnow();
+    ds_split<K, V>(R, sl, sr, A, B);
+    if (tid == 0) {
+      R.tacc(3, t3);
+      const u32 x = c->b[5], y = c->b[6], up = c->b[9], minc = c->b[13], l = c->b[11], r = c->b[12];
+      const ull t4 = R.tnow();
+      const DsMsg b = R.recv();
+      R.tacc(4, t4);
+      asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+      R.release(push_old);
+      push_old = DS_NONE;
+      c->b[14] = 0;
+      if (b.kind == MK_BSTOP || b.cmax <= minc) {  // stopped above / at cur: nothing changes below
+        if (b.kind != MK_BSTOP) {                  // cur keeps the carried keys
+          const u32 s = R.alloc();
+          R.load_node(s, b.src);
+          R.push_up(s, up);
+          push_old = s;
+        }
+        sq_req<K, V>(R, &c->wq_head, &c->wq_done, c->wq, WQ_CANCEL, y, l, r, 0);
+        R.release(A); R.release(B);
+        st_rel_cta(&c->sq_ret, (u32)i + 1u);
+      } else {
+        c->st[S_DEL_LEVELS]++;
+        c->st[c->b[10] ? S_DEL_LR_NOMOVE : S_DEL_LR_MERGE]++;
+        st_rel_cta(&c->sq_ret, (u32)i + 1u);  // the staged children were only split inputs
+        // x <- X: HBM write-back, then UNLOCK(x) (helper B, l.11); it frees slot B
+        sq_req<K, V>(R, &c->wq_head, &c->wq_done, c->wq, WQ_WB, x, B, R.BK(B)[0], R.BK(B)[K - 1]);
+        const u32 ymax = R.BK(A)[K - 1];
+        if (ymax <= b.cmin) {  // l.12 swap: cur <- Y, the carried keys go on to y's walker
+          c->st[S_DEL_CY_SWAP]++;
+          R.push_up(A, up);
+          push_old = A;
+          sq_req<K, V>(R, &c->wq_head, &c->wq_done, c->wq, WQ_COMMIT, y, b.src, 0, 0);
+        } else {
+          const u32 cs = R.alloc(), lo = R.alloc(), hi = R.alloc();
+          R.load_node(cs, b.src);
+          c->b[14] = 1; c->b[4] = cs; c->b[5] = lo; c->b[6] = hi; c->b[7] = y; c->b[9] = up; c->b[12] = A;
+        }
+      }
+    }
+    cta_bar<DS_NT>();
+    if (c->b[14]) {  // rare: a real (cur, y) merge
+      const u32 cs = c->b[4], lo = c->b[5], hi = c->b[6], Y = c->b[12];
+      ds_split<K, V>(R, cs, Y, lo, hi);
+      if (tid == 0) {
+        const u32 y = c->b[7], up = c->b[9];
+        R.store_node(y, hi);  // the carried keys in y's HBM copy (y is LOCKed by us)
+        __threadfence();
+        R.push_up(lo, up);
+        push_old = lo;
+        R.release(cs); R.release(Y); R.release(hi);
+        sq_req<K, V>(R, &c->wq_head, &c->wq_done, c->wq, WQ_COMMIT, y, y, 0, 0);
+      }
+      cta_bar<DS_NT>();
+    }
+    if (tid == 0) {  // slots the write-back helper finished with
+      const u32 fr = atomicExch(&c->wb_free, 0u);
+      R.fm |= fr;
+    }
+  }
+  if (tid == 0) {
+    R.tacc(0, t_start);
+    asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+  }
+}
+
+// stager helper A (lane 0 of warp DS_NT/32): reads the path messages "a" from the second inbox
+// as they arrive (up to 4 ops ahead of thread 0), LOCKs and stages the two children of each
+// path node (in op order) into its own slot ring, and publishes one record per op.
+template <int K, bool V>
+__device__ void ds_stage_helper(DsRole<K, V>& R, const u64 m) {
+  DsCtl* c = R.c;
+  const HeapArgs& H = R.H;
+  for (u32 k = 0; k < (u32)m; ++k) {
+    const u32 e = k % DS_RING;
+    mbar_wait(&c->ainbar[e], (k / DS_RING) & 1u);
+    const u32 kind = c->ainbox[e].kind, y = c->ainbox[e].y, up = c->ainbox[e].slot;
+    mbar_arrive_expect_tx(&c->ainbar[e], (u32)sizeof(DsMsg));  // re-arm
+    if ((k + 1) % DS_CREDIT == 0)
+      asm volatile("st.relaxed.cluster.shared::cluster.u32 [%0], %1;" ::"r"(cl_map(&c->aconsumed, R.rank - 1)),
+                   "r"(k + 1) : "memory");
+    const u32 q = k % 16;
+    while (k >= ld_acq_cta(&c->sq_ret) + 4u) {}  // op k - 4 done: its record and staging slots are free
+    if (kind == MK_ASTOP) {
+      c->stg_y[q] = 0;
+    } else {
+      const u32 n0 = 2u * y, n1 = n0 + 1u;
+      const u32 s0 = DS_NSLOT - 8 + 2 * (k % 4), s1 = s0 + 1;
+      lock_acquire(&H.meta[n0].lock);  // l.3: LOCK(l); LOCK(r)
+      lock_acquire(&H.meta[n1].lock);
+      fence_proxy_async();
+      u64* bar = &c->sbar[k % 4];  // thread 0 waits for the data; this helper moves on
+      mbar_arrive_expect_tx(bar, 2u * DsRole<K, V>::SLOTB);
+      bulk_g2s(R.BK(s0), H.gk + (size_t)n0 * K, DsRole<K, V>::NB, bar);
+      bulk_g2s(R.BK(s1), H.gk + (size_t)n1 * K, DsRole<K, V>::NB, bar);
+      if (V) {
+        bulk_g2s(R.BV(s0), H.gv + (size_t)n0 * K, DsRole<K, V>::NB, bar);
+        bulk_g2s(R.BV(s1), H.gv + (size_t)n1 * K, DsRole<K, V>::NB, bar);
+      }
+      c->stg_min[q][0] = ld_relaxed(&H.meta[n0].kmin); c->stg_max[q][0] = ld_relaxed(&H.meta[n0].kmax);
+      c->stg_min[q][1] = ld_relaxed(&H.meta[n1].kmin); c->stg_max[q][1] = ld_relaxed(&H.meta[n1].kmax);
+      c->stg_y[q] = y;
+      c->stg_up[q] = up;
+    }
+    st_rel_cta(&c->sq_done, k + 1u);
+  }
+}
+
+// stager helper B (lane 0 of warp DS_NT/32 + 1): walker tasks, write-backs, UNLOCKs
+template <int K, bool V>
+__device__ void ds_wb_helper(DsRole<K, V>& R) {
+  DsCtl* c = R.c;
+  const HeapArgs& H = R.H;
+  u32 seen = 0, tasks = 0, go_next = 0;
+  for (;;) {
+    const u32 head = ld_acq_cta(&c->wq_head);
+    if (seen == head) {
+      if (ld_acq_cta(&c->quit)) break;
+      continue;
+    }
+    const u32* e = c->wq + (seen % 16) * 5;
+    const u32 kind = e[0];
+    if (kind == WQ_PUBLISH) {  // y is LOCKed (staged by helper A): task visible, carried keys later
+      st_relaxed(R.D.task_node + tasks, e[1]);
+      st_release(R.D.task_seq + tasks, R.D.epoch);
+      ++tasks;
+    } else if (kind == WQ_COMMIT || kind == WQ_CANCEL) {
+      // a merged carried set was stored to HBM by thread 0 (wait_group + __threadfence) before
+      // its request, which this thread acquired
+      const u32 t = go_next++;
+      st_release_u64(R.D.task_go + t, ((u64)R.D.epoch << 32) | (kind == WQ_COMMIT ? e[2] : 0xFFFFFFFFu));
+      if (kind == WQ_CANCEL) {  // y and its sibling stay as they were: UNLOCK both
+        asm volatile("fence.acq_rel.gpu;" ::: "memory");
+        st_relaxed(&H.meta[e[2]].lock, 0u);
+        st_relaxed(&H.meta[e[3]].lock, 0u);
+      }
+    } else if (kind == WQ_WB) {  // Alg.3 l.10-11: x <- X, UNLOCK(x)
+      const u32 x = e[1], B = e[2];
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      bulk_s2g(H.gk + (size_t)x * K, R.BK(B), DsRole<K, V>::NB);
+      if (V) bulk_s2g(H.gv + (size_t)x * K, R.BV(B), DsRole<K, V>::NB);
+      asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+      asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+      st_relaxed(&H.meta[x].kmin, e[3]);
+      st_relaxed(&H.meta[x].kmax, e[4]);
+      asm volatile("fence.proxy.async.global;" ::: "memory");
+      asm volatile("fence.acq_rel.gpu;" ::: "memory");
+      st_relaxed(&H.meta[x].lock, 0u);
+      atomicOr(&c->wb_free, 1u << B);
+    }
+    ++seen;
+    st_rel_cta(&c->wq_done, seen);
+  }
+  st_release(R.D.ctl + 1, tasks + 1u);  // walkers: the final task count
+}
+
+template <int K, bool V>
+__global__ void __cluster_dims__(DS_CL, 1, 1) __launch_bounds__(DS_BLOCK, 1)
+    bgpq_dsys_kernel(HeapArgs H, CallArgs C, DtArgs D) {
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  const u64 m = ds_ops(H, C, K);
+  if (blockIdx.x < DS_CL) {
+    DsCtl* c = reinterpret_cast<DsCtl*>(smem_raw);
+    DsRole<K, V> R;
+    R.H = H; R.C = C; R.D = D; R.c = c;
+    R.sk = reinterpret_cast<u32*>(smem_raw + DSCTL_BYTES);
+    R.sv = R.sk + DS_NSLOT * K;
+    R.rank = cl_rank();
+    // the stager keeps its last 8 slots for staging (helper A's ring)
+    R.fm = (R.rank == DS_CL - 1) ? ((1u << (DS_NSLOT - 8)) - 1u) : ((1u << DS_NSLOT) - 1u);
+    R.sbph = 0; R.in_seq = 0; R.out_seq = 0; R.out_seq2 = 0; R.lph = 0;
+    R.timing = (C.debug & 1024u) != 0;
+    if (threadIdx.x == 0) {
+      for (u32 e = 0; e < DS_RING; ++e) mbar_init(&c->inbar[e], 1);
+      for (u32 e = 0; e < DS_RING; ++e) R.arm_inbox(e);
+      for (u32 s = 0; s < DS_NSLOT; ++s) mbar_init(&c->slotbar[s], 1);
+      mbar_init(&c->lbar, 1);
+      mbar_init(&c->hbar, 1);
+      for (int q = 0; q < 4; ++q) mbar_init(&c->sbar[q], 1);
+      c->consumed = 0; c->rf_seq = 0; c->rf_used = 0; c->tasks = 0; c->quit = 0;
+      c->sq_done = 0; c->sq_ret = 0; c->wq_head = 0; c->wq_done = 0; c->wb_free = 0; c->aconsumed = 0;
+      for (u32 e = 0; e < DS_RING; ++e) {
+        mbar_init(&c->ainbar[e], 1);
+        mbar_arrive_expect_tx(&c->ainbar[e], (u32)sizeof(DsMsg));
+      }
+      for (int q = 0; q < NSTAT; ++q) c->st[q] = 0;
+      for (int q = 0; q < 8; ++q) c->tm[q] = 0;
+      asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    cluster_sync_all();  // every barrier of the cluster initialised before any remote copy
+    const bool stager = R.rank == DS_CL - 1;
+    if (threadIdx.x >= DS_NT) {
+      if (threadIdx.x == DS_NT) {
+        if (R.rank == 0) ds_r0_helper<K, V>(R, m);
+        else if (stager) ds_stage_helper<K, V>(R, m);
+      } else if (threadIdx.x == DS_NT + 32 && stager) {
+        ds_wb_helper<K, V>(R);
+      }
+    } else {
+      if (m) {
+        if (R.rank == 0) ds_r0<K, V>(R, m);
+        else if (stager) ds_stager<K, V>(R, m);
+        else ds_level<K, V>(R, m);
+      } else if (threadIdx.x == 0 && R.rank == 0) {
+        *reinterpret_cast<volatile u64*>(D.op_base) = 0;
+      }
+      cta_bar<DS_NT>();
+      if (threadIdx.x == 0) st_rel_cta(&c->quit, 1u);
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      ull* stat = reinterpret_cast<ull*>(H.hdr + H_STAT);
+      for (int q = 0; q < NSTAT; ++q)
+        if (c->st[q]) atomicAdd(stat + q, c->st[q]);
+      if (R.timing) {
+        ull* tms = reinterpret_cast<ull*>(H.hdr + H_TIME);
+        for (int q = 0; q < 6; ++q) atomicAdd(tms + 6 * R.rank + q, c->tm[q]);
+      }
+    }
+    cluster_sync_all();  // no CTA leaves while a peer may still access its shared memory
+    return;
+  }
+  dt_walkers<K, V, DS_NT>(H, C, D, smem_raw);
+}
+
+}  // namespace bgpqd

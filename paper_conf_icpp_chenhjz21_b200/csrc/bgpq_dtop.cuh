@@ -49,10 +49,14 @@ constexpr u32 DT_BIG = 64;              // pipelined mode needs heapSize >= DT_B
 constexpr u32 DT_NONE = 0xFFFFFFFFu;
 
 struct DtArgs {
-  u32* task_node;  // [cap_nodes + 2]: node handed to a walker (locked, content in HBM)
-  u32* task_seq;   // [cap_nodes + 2]: call epoch once task_node is valid (release)
+  u32* task_node;  // [cap_nodes + 2 + grid]: node handed to a walker (locked, content in HBM)
+  u32* task_seq;   // [cap_nodes + 2 + grid]: call epoch once task_node is valid (release)
+  u64* task_go;    // [cap_nodes + 2 + grid]: (epoch << 32) | node whose HBM copy holds the
+                   // carried keys, or | 0xFFFFFFFF: cancelled (published early, walk stopped above)
   u32* ctl;        // [0] walker ticket, [1] final task count + 1 (release), reset per call
-  u32 epoch;       // per call, >= 1
+  u64* op_base;    // nullable: ops of this call already executed by the cluster engine
+                   // (bgpq_dsys.cuh); this launch executes the rest
+  u32 epoch;       // per launch, >= 1
 };
 
 enum : u32 { RQ_STAGE = 1, RQ_REFILL = 2, RQ_WB = 3, RQ_END = 4, RQ_WB2 = 5 };
@@ -413,6 +417,7 @@ __device__ __forceinline__ void dt_helper(DTop<K, V>& T, const u32 hr) {
         if (e[3]) {
           const u32 t = c->tasks++;
           st_relaxed(T.D.task_node + t, e[3]);
+          st_relaxed_u64(T.D.task_go + t, ((u64)T.D.epoch << 32) | e[3]);
           st_release(T.D.task_seq + t, T.D.epoch);
         }
       } else if (type == RQ_WB2) {  // Alg.3 l.10-15 write-backs of the lag step, then UNLOCK / hand over
@@ -436,6 +441,7 @@ __device__ __forceinline__ void dt_helper(DTop<K, V>& T, const u32 hr) {
         if (fl2 & 1u) {
           const u32 t = c->tasks++;
           st_relaxed(T.D.task_node + t, y);
+          st_relaxed_u64(T.D.task_go + t, ((u64)T.D.epoch << 32) | y);
           st_release(T.D.task_seq + t, T.D.epoch);
         } else {
           st_relaxed(T.lk(y), 0u);
@@ -1251,21 +1257,46 @@ __device__ __forceinline__ void dt_top(DTop<K, V>& T) {
 // keys stored in the node), with OpL's lock-ahead agents (bgpq_locks.cuh).
 // =========================================================================================
 template <int K, bool V, int NT>
-__device__ void dt_walk(OpL<K, V, NT>& op, u32 cur) {
+__device__ void dt_walk(OpL<K, V, NT>& op, u32 cur, const u64* go, u32 epoch, ull* wtm = nullptr) {
+  ull t_go = 0;
+  bool first = true;
   const int tid = threadIdx.x;
   LCtl* ctl = op.ctl;
   if (tid == 0) {
     const u32 l = 2u * cur, r = l + 1u;
     const u32 n0 = l <= op.H.cap ? l : 0u, n1 = r <= op.H.cap ? r : 0u;
     const int s0 = op.alloc(), s1 = op.alloc();
-    op.post_p(n0, n1, s0, s1, 0u);
+    op.post_p(n0, n1, s0, s1, 0u);  // LOCK + stage the children while the hand-over completes
     ctl->b[8] = (u32)s0; ctl->b[9] = (u32)s1;
     ctl->b[10] = (u32)op.alloc();
+    // the task may have been published before its carried keys were final: wait for them
+    u64 g;
+    u32 ns = 32;
+    for (;;) {
+      asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(g) : "l"(go) : "memory");
+      if ((u32)(g >> 32) == epoch) break;
+      __nanosleep(ns);
+      ns = ns < 256 ? ns * 2 : 256;
+    }
+    ctl->b[11] = (u32)g;
+    if (wtm) t_go = clock64();
   }
   cta_bar<NT>();
   int R = (int)ctl->b[10];
   int SL = (int)ctl->b[8], SRr = (int)ctl->b[9];
-  op.load(R, cur);  // the carried keys (written by the top CTA before the hand-over)
+  const u32 src = ctl->b[11];
+  if (src == 0xFFFFFFFFu) {  // cancelled: the walk stopped above this node — release the children
+    op.wait_p(LT_DEL_PWAIT);
+    if (tid == 0) {
+      const u32 l = 2u * cur, r = l + 1u;
+      if (l <= op.H.cap) lock_release(op.lk(l));
+      if (r <= op.H.cap) lock_release(op.lk(r));
+      op.free_slot(SL); op.free_slot(SRr); op.free_slot(R);
+    }
+    cta_bar<NT>();
+    return;
+  }
+  op.load(R, src);  // the carried keys (in cur's HBM copy, or in the refill node they came from)
   for (;;) {
     const u32 l = 2u * cur, r = l + 1u;
     op.wait_p(LT_DEL_PWAIT);  // l.3: LOCK(l); LOCK(r), children staged
@@ -1358,6 +1389,7 @@ __device__ void dt_walk(OpL<K, V, NT>& op, u32 cur) {
       op.set_minmax(cur, op.BK(C2)[0], op.BK(C2)[K - 1]);
       op.free_slot(C2);
       op.release_locks(cur, ctl->b[16]);  // l.14 (and l.11)
+      if (wtm && first) { wtm[0] += clock64() - t_go; wtm[1] += 1; first = false; }
     }
     cur = y;  // l.15
     R = Y2;
@@ -1376,9 +1408,86 @@ __device__ void dt_walk(OpL<K, V, NT>& op, u32 cur) {
   }
 }
 
+// Walker CTAs: take tasks (a depth-3 node handed over locked + the node holding its carried
+// keys) by ticket and run Alg.3 from l.2 below it (dt_walk), until the final count is published.
+template <int K, bool V, int NT>
+__device__ __forceinline__ void dt_walkers(const HeapArgs& H, const CallArgs& C, const DtArgs& D,
+                                           unsigned char* smem_raw) {
+  LCtl* ctl = reinterpret_cast<LCtl*>(smem_raw);
+  OpL<K, V, NT> op;
+  op.H = H;
+  op.ctl = ctl;
+  op.sk = reinterpret_cast<u32*>(smem_raw + LCTL_BYTES);
+  op.sv = op.sk + LSLOT * K;
+  op.mphase = 0; op.pph = 0; op.tphase = 0; op.pb = 0;
+  op.st = ctl->st;
+  op.tm = ctl->tm;
+  op.timing = false;
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < NSTAT; ++i) ctl->st[i] = 0;
+    ctl->tm[28] = 0; ctl->tm[29] = 0;
+    mbar_init(&ctl->bar, 1);
+    mbar_init(&ctl->pbar[0], 1);
+    mbar_init(&ctl->pbar[1], 1);
+    mbar_init(&ctl->tbar, 1);
+    ctl->freemask = (1u << LSLOT) - 1u;
+    ctl->p_req = 0; ctl->t_req = 0; ctl->t_done = 0; ctl->stop = 0; ctl->t_marked = 0;
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  if (threadIdx.x >= NT) {
+    if (threadIdx.x < NT + 32) lock_warp<K, V, NT>(op);
+    return;
+  }
+  for (;;) {
+    if (threadIdx.x == 0) {
+      const u32 t = atomicAdd(D.ctl, 1u);
+      u32 node = 0, ns = 32, k = 0;
+      for (;;) {
+        if (ld_acquire(D.task_seq + t) == D.epoch) {
+          node = ld_relaxed(D.task_node + t);
+          break;
+        }
+        if ((++k & 7u) == 0) {
+          const u32 fin = ld_acquire(D.ctl + 1);
+          if (fin && t + 1u >= fin) break;
+        }
+        __nanosleep(ns);
+        ns = ns < 512 ? ns * 2 : 512;
+      }
+      ctl->b[0] = node;
+      ctl->b[1] = t;
+    }
+    cta_bar<NT>();
+    const u32 node = ctl->b[0], tk = ctl->b[1];
+    cta_bar<NT>();
+    if (threadIdx.x == 0 && C.prog && blockIdx.x < 500) C.prog[16 + 2 * blockIdx.x] = node;
+    if (!node) break;
+    dt_walk<K, V, NT>(op, node, D.task_go + tk, D.epoch, (C.debug & 1024u) ? &ctl->tm[28] : nullptr);
+  }
+  if (threadIdx.x == 0) {
+    st_rel_cta(&ctl->stop, 1u);
+    ull* stat = reinterpret_cast<ull*>(H.hdr + H_STAT);
+    for (int i = 0; i < NSTAT; ++i)
+      if (op.st[i]) atomicAdd(stat + i, op.st[i]);
+    if (C.debug & 1024u) {  // walker first-level hold time (go -> release of the start node)
+      ull* tms = reinterpret_cast<ull*>(H.hdr + H_TIME);
+      atomicAdd(tms + 30, ctl->tm[28]);
+      atomicAdd(tms + 31, ctl->tm[29]);
+    }
+  }
+}
+
 template <int K, bool V>
 __global__ void __launch_bounds__(DT_BLOCK, 1) bgpq_dtop_kernel(HeapArgs H, CallArgs C, DtArgs D) {
   extern __shared__ __align__(128) unsigned char smem_raw[];
+  if (D.op_base) {  // the cluster engine executed the first ops of the call: continue after them
+    const u64 b = *reinterpret_cast<volatile const u64*>(D.op_base);
+    C.n -= b * (u64)K;
+    C.n_ops -= b;
+    C.out_k += b * (u64)K;
+    if (C.out_v) C.out_v += b * (u64)K;
+  }
   if (blockIdx.x == 0) {
     DtCtl* c = reinterpret_cast<DtCtl*>(smem_raw);
     DTop<K, V> T;
@@ -1406,60 +1515,7 @@ __global__ void __launch_bounds__(DT_BLOCK, 1) bgpq_dtop_kernel(HeapArgs H, Call
     dt_top<K, V>(T);
     return;
   }
-  // ---- walkers
-  LCtl* ctl = reinterpret_cast<LCtl*>(smem_raw);
-  OpL<K, V, DT_NTC> op;
-  op.H = H;
-  op.ctl = ctl;
-  op.sk = reinterpret_cast<u32*>(smem_raw + LCTL_BYTES);
-  op.sv = op.sk + LSLOT * K;
-  op.mphase = 0; op.pph = 0; op.tphase = 0; op.pb = 0;
-  op.st = ctl->st;
-  op.tm = ctl->tm;
-  op.timing = false;
-  if (threadIdx.x == 0) {
-    for (int i = 0; i < NSTAT; ++i) ctl->st[i] = 0;
-    mbar_init(&ctl->bar, 1);
-    mbar_init(&ctl->pbar[0], 1);
-    mbar_init(&ctl->pbar[1], 1);
-    mbar_init(&ctl->tbar, 1);
-    ctl->freemask = (1u << LSLOT) - 1u;
-    ctl->p_req = 0; ctl->t_req = 0; ctl->t_done = 0; ctl->stop = 0; ctl->t_marked = 0;
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-  }
-  __syncthreads();
-  if (threadIdx.x >= DT_NTC) {
-    if (threadIdx.x < DT_NTC + 32) lock_warp<K, V, DT_NTC>(op);
-    return;
-  }
-  for (;;) {
-    if (threadIdx.x == 0) {
-      const u32 t = atomicAdd(D.ctl, 1u);
-      u32 node = 0, ns = 32, k = 0;
-      for (;;) {
-        if (ld_acquire(D.task_seq + t) == D.epoch) { node = ld_relaxed(D.task_node + t); break; }
-        if ((++k & 7u) == 0) {
-          const u32 fin = ld_acquire(D.ctl + 1);
-          if (fin && t + 1u >= fin) break;
-        }
-        __nanosleep(ns);
-        ns = ns < 512 ? ns * 2 : 512;
-      }
-      ctl->b[0] = node;
-    }
-    cta_bar<DT_NTC>();
-    const u32 node = ctl->b[0];
-    cta_bar<DT_NTC>();
-    if (threadIdx.x == 0 && C.prog && blockIdx.x < 500) C.prog[16 + 2 * blockIdx.x] = node;
-    if (!node) break;
-    dt_walk<K, V, DT_NTC>(op, node);
-  }
-  if (threadIdx.x == 0) {
-    st_rel_cta(&ctl->stop, 1u);
-    ull* stat = reinterpret_cast<ull*>(H.hdr + H_STAT);
-    for (int i = 0; i < NSTAT; ++i)
-      if (op.st[i]) atomicAdd(stat + i, op.st[i]);
-  }
+  dt_walkers<K, V, DT_NTC>(H, C, D, smem_raw);
 }
 
 }  // namespace bgpqd

@@ -34,6 +34,22 @@ cudaError_t dt_launch(int grid, const HeapArgs& H, const CallArgs& C, const DtAr
   bgpq_dtop_kernel<K, V><<<grid, DT_BLOCK, dt_smem_bytes<K, V>(), s>>>(H, C, D);
   return cudaGetLastError();
 }
+cudaError_t ds_prepare(int sm_count, int* clusters) {
+  *clusters = 0;
+  auto kern = bgpq_dsys_kernel<K, V>;
+  const size_t smem = ds_smem_bytes<K, V>();
+  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((sm_count / DS_CL) * DS_CL);
+  cfg.blockDim = dim3(DS_BLOCK);
+  cfg.dynamicSmemBytes = smem;
+  return cudaOccupancyMaxActiveClusters(clusters, kern, &cfg);
+}
+cudaError_t ds_launch(int grid, const HeapArgs& H, const CallArgs& C, const DtArgs& D, cudaStream_t s) {
+  bgpq_dsys_kernel<K, V><<<grid, DS_BLOCK, ds_smem_bytes<K, V>(), s>>>(H, C, D);
+  return cudaGetLastError();
+}
 cudaError_t pipe_prepare(int* occ) {
   auto kern = bgpq_ins_pipe2_kernel<K, V, NT>;
   const size_t smem = pipe2_smem_bytes<K, V>();
@@ -46,7 +62,8 @@ cudaError_t pipe_launch(int grid, const HeapArgs& H, const PipeArgs& P, const Ca
   return cudaGetLastError();
 }
 
-const KTable kTable = {locks_prepare, locks_launch, dt_prepare, dt_launch, pipe_prepare, pipe_launch};
+const KTable kTable = {locks_prepare, locks_launch, dt_prepare, dt_launch, ds_prepare, ds_launch, pipe_prepare,
+                       pipe_launch};
 
 }  // namespace
 

@@ -6,6 +6,7 @@
 #include <cuda_runtime.h>
 
 #include "bgpq_dtop.cuh"
+#include "bgpq_dsys.cuh"
 #include "bgpq_pipe2.cuh"
 
 namespace bgpqd {
@@ -20,6 +21,10 @@ struct KTable {
   // deletemin calls: top CTA + walkers (bgpq_dtop.cuh)
   cudaError_t (*dt_prepare)(int* occ);
   cudaError_t (*dt_launch)(int grid, const HeapArgs& H, const CallArgs& C, const DtArgs& D, cudaStream_t s);
+  // deletemin calls, steady state: 3-CTA cluster + walkers (bgpq_dsys.cuh); prepare returns
+  // the number of co-resident clusters in *clusters (0 if the engine cannot run)
+  cudaError_t (*ds_prepare)(int sm_count, int* clusters);
+  cudaError_t (*ds_launch)(int grid, const HeapArgs& H, const CallArgs& C, const DtArgs& D, cudaStream_t s);
   // insert calls: level pipeline (bgpq_pipe2.cuh)
   cudaError_t (*pipe_prepare)(int* occ);
   cudaError_t (*pipe_launch)(int grid, const HeapArgs& H, const PipeArgs& P, const CallArgs& C, cudaStream_t s);
