@@ -288,10 +288,12 @@ __device__ __forceinline__ void ds_split(DsRole<K, V>& R, u32 z, u32 w, u32 x, u
 }
 
 // Number of full-K ops the engine executes (identical in every role CTA): the call's full
-// batches, while heapSize stays >= DS_HMIN, if |root| = K and the pBuffer is empty.
+// batches, while heapSize stays >= DS_HMIN, if |root| is K or 0 and the pBuffer is empty.
+// (|root| = 0 is the state a drained heap keeps, reading R4: then every DELETEMIN refills the
+// root and extracts all K keys of it after the heapify, Alg.2 l.4-14 + l.5-6 of Alg.3.)
 __device__ __forceinline__ u64 ds_ops(const HeapArgs& H, const CallArgs& C, int K) {
   const u32 hs = ld_relaxed(H.hdr + H_HS), rs = ld_relaxed(H.hdr + H_RS), ps = ld_relaxed(H.hdr + H_PS);
-  if (rs != (u32)K || ps != 0 || hs < DS_HMIN + 2) return 0;
+  if ((rs != (u32)K && rs != 0) || ps != 0 || hs < DS_HMIN + 2) return 0;
   const u64 full = C.n / (u64)K;
   const u64 room = hs - DS_HMIN;
   return full < room ? full : room;
@@ -306,21 +308,27 @@ __device__ void ds_r0(DsRole<K, V>& R, const u64 m) {
   const HeapArgs& H = R.H;
   const int tid = threadIdx.x;
   u32 hs = ld_relaxed(H.hdr + H_HS);
+  // |root| = K: op i outputs the root (Alg.2 l.22) and refills it; |root| = 0 (R4): op i
+  // refills the empty root and extracts all K keys after the heapify (l.14 + Alg.3 l.5-6),
+  // so it outputs the root's new content and leaves it empty
+  const bool rz = ld_relaxed(H.hdr + H_RS) == 0;
   // on-chip nodes: 1 (root), 2, 3
   u32* ns = c->ns;
   u32* mn = c->mn;
   u32* mx = c->mx;
   u32* pend = c->pend;
   if (tid == 0) {
-    for (u32 q = 1; q <= 3; ++q) {
+    ns[1] = DS_NONE;
+    for (u32 q = rz ? 2 : 1; q <= 3; ++q) {
       ns[q] = R.alloc();
       pend[q] = 0;
       mn[q] = ld_relaxed(&H.meta[q].kmin);
       mx[q] = ld_relaxed(&H.meta[q].kmax);
     }
+    pend[1] = 0;
     fence_proxy_async();
-    mbar_arrive_expect_tx(&c->lbar, 3u * DsRole<K, V>::SLOTB);
-    for (u32 q = 1; q <= 3; ++q) {
+    mbar_arrive_expect_tx(&c->lbar, (rz ? 2u : 3u) * DsRole<K, V>::SLOTB);
+    for (u32 q = rz ? 2 : 1; q <= 3; ++q) {
       bulk_g2s(R.BK(ns[q]), H.gk + (size_t)q * K, DsRole<K, V>::NB, &c->lbar);
       if (V) bulk_g2s(R.BV(ns[q]), H.gv + (size_t)q * K, DsRole<K, V>::NB, &c->lbar);
     }
@@ -328,7 +336,18 @@ __device__ void ds_r0(DsRole<K, V>& R, const u64 m) {
     R.lph ^= 1u;
   }
   cta_bar<DS_NT>();
-  u32 out_old = DS_NONE;  // root slot whose output store may still be reading it
+  u32 out_old = DS_NONE;  // slot whose output store may still be reading it
+  // op i's K output keys from slot s (TMA bulk store; the slot is freed once it was read)
+  auto output = [&](u64 i, u32 s) {
+    asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");  // the previous output's read
+    R.release(out_old);
+    const u64 pos = i * (u64)K;
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    bulk_s2g(R.C.out_k + pos, R.BK(s), DsRole<K, V>::NB);
+    if (V && R.C.out_v) bulk_s2g(R.C.out_v + pos, R.BV(s), DsRole<K, V>::NB);
+    asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+    out_old = s;
+  };
   const ull t_start = R.tnow();
   for (u64 i = 0; i < m; ++i) {
     if (tid == 0) {
@@ -350,23 +369,16 @@ __device__ void ds_r0(DsRole<K, V>& R, const u64 m) {
           mx[q] = R.BK(ns[q])[K - 1];
         }
       R.tacc(2, t2);
-      // Alg.2 l.22: the root's K keys are op i's output (TMA bulk store, async)
-      asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");  // the previous output's read
-      R.release(out_old);
-      const u64 pos = i * (u64)K;
-      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-      bulk_s2g(R.C.out_k + pos, R.BK(ns[1]), DsRole<K, V>::NB);
-      if (V && R.C.out_v) bulk_s2g(R.C.out_v + pos, R.BV(ns[1]), DsRole<K, V>::NB);
-      asm volatile("cp.async.bulk.commit_group;" ::: "memory");
-      out_old = ns[1];
+      if (!rz) output(i, ns[1]);  // Alg.2 l.22: the root's K keys are op i's output
       c->st[S_DEL_OPS]++;
       c->st[S_DEL_REFILL]++;
-      // Alg.3 at the root: cur = root holding the refill keys (R3: |root| = K = size refills)
+      // Alg.3 at the root: cur = root holding the refill keys
       const u32 minc = mn[2] < mn[3] ? mn[2] : mn[3];
       if (rmax <= minc) {  // l.4: stop at the root — root <- the refill keys
         const u32 s = R.alloc();
         R.load_node(s, t);
-        ns[1] = s; mn[1] = rmin; mx[1] = rmax;
+        if (rz) output(i, s);
+        else { ns[1] = s; mn[1] = rmin; mx[1] = rmax; }
         R.send((u32)i, MK_ASTOP);
         c->b[0] = 1;
       } else {
@@ -392,17 +404,19 @@ __device__ void ds_r0(DsRole<K, V>& R, const u64 m) {
       R.release(s2); R.release(s3);
       const u32 ymax = R.BK(A)[K - 1];
       if (ymax <= rmin) {  // l.12 is a swap: root <- Y, the refill keys sink on (by reference)
-        ns[1] = A; mn[1] = R.BK(A)[0]; mx[1] = ymax;
         c->st[S_DEL_CY_SWAP]++;
         R.send((u32)i, MK_B, 0, 0, t, rmin, rmax);
+        if (rz) output(i, A);  // Alg.3 l.5-6 / l.13: the root's new keys are extracted
+        else { ns[1] = A; mn[1] = R.BK(A)[0]; mx[1] = ymax; }
+        c->b[15] = 0;
       } else {  // l.12 merges: (root, C1) <- SORT_SPLIT(refill, Y); C1 into y1's dead HBM copy
         const u32 r = R.alloc(), lo = R.alloc(), hi = R.alloc();
         R.load_node(r, t);
-        c->b[11] = r; c->b[12] = lo; c->b[13] = hi; c->b[14] = 1;
+        c->b[11] = r; c->b[12] = lo; c->b[13] = hi;
+        c->b[15] = 1;
       }
       ns[x] = B; mn[x] = R.BK(B)[0]; mx[x] = R.BK(B)[K - 1];
       ns[y] = sy; pend[y] = 1;
-      if (!(ymax <= rmin)) c->b[15] = 1; else c->b[15] = 0;
     }
     cta_bar<DS_NT>();
     if (c->b[15]) {  // rare: a real (cur, y) merge at the root
@@ -413,7 +427,8 @@ __device__ void ds_r0(DsRole<K, V>& R, const u64 m) {
         R.store_node(y, hi);  // C1 in y1's HBM copy (y1 is on chip; its HBM copy is dead)
         __threadfence();
         R.send((u32)i, MK_B, 0, 0, y, R.BK(hi)[0], R.BK(hi)[K - 1]);
-        ns[1] = lo; mn[1] = R.BK(lo)[0]; mx[1] = R.BK(lo)[K - 1];
+        if (rz) output(i, lo);
+        else { ns[1] = lo; mn[1] = R.BK(lo)[0]; mx[1] = R.BK(lo)[K - 1]; }
         R.release(r); R.release(hi); R.release(A);
       }
       cta_bar<DS_NT>();
@@ -425,7 +440,7 @@ __device__ void ds_r0(DsRole<K, V>& R, const u64 m) {
     for (u32 q = 2; q <= 3; ++q)
       if (pend[q]) { R.wait_pushed(ns[q]); pend[q] = 0; mn[q] = R.BK(ns[q])[0]; mx[q] = R.BK(ns[q])[K - 1]; }
     asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
-    for (u32 q = 1; q <= 3; ++q) {
+    for (u32 q = rz ? 2 : 1; q <= 3; ++q) {
       R.store_node(q, ns[q]);
       st_relaxed(&H.meta[q].kmin, mn[q]);
       st_relaxed(&H.meta[q].kmax, mx[q]);
@@ -437,7 +452,6 @@ __device__ void ds_r0(DsRole<K, V>& R, const u64 m) {
     c->st[S_KEYS_OUT] += m * (u64)K;
     if (R.C.d_count && m) atomicAdd(R.C.d_count, (ull)(m * (u64)K));
     *reinterpret_cast<volatile u64*>(R.D.op_base) = m;
-    c->quit = 1;
   }
 }
 

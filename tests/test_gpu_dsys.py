@@ -119,3 +119,26 @@ def test_cluster_engine_disabled_switch_same_output():
         finally:
             pkg.set_debug(0)
     assert np.array_equal(outs[0], outs[1]) and np.array_equal(outs[0], np.sort(keys))
+
+
+@pytest.mark.parametrize("K,values", [(1024, False), (256, True)])
+def test_cluster_engine_reused_heap_root_empty(K, values):
+    """After a full drain the heap keeps heapSize = 1 with an empty root (R4); the next insert
+    call leaves |root| = 0 and every DELETEMIN then refills the root and extracts all K keys
+    after the heapify (Alg.2 l.4-14, Alg.3 l.5-6 / l.13).  The engine runs in that regime too."""
+    n = 1500 * K + 3
+    q = pkg.BGPQ(capacity=n, K=K, values=values)
+    for rep in range(3):
+        keys = synth.keys(n, seed=70 + rep, dist="uniform" if rep != 1 else "dups")
+        q.insert(_dev(keys), _dev(synth.values(n)) if values else None)
+        if rep:
+            assert q.dump()[3]["rootSize"] == 0
+        l0 = pkg.launch_count()
+        ok, ov = q.deletemin(n)
+        assert pkg.launch_count() - l0 == 2
+        out = _host(ok)
+        assert np.array_equal(out, np.sort(keys)), rep
+        if values:
+            assert np.array_equal(keys[_host(ov)], out)
+        assert q.size() == 0
+    q.close()
