@@ -24,6 +24,7 @@ namespace bgpqd {
 
 constexpr u32 P2_PIN = 4;     // in-ring entries (H1 -> compute)
 constexpr u32 P2_RQ = 16;     // H2 request ring
+constexpr u32 P2_H2D = 4;     // H2 requests in flight (bulk groups)
 constexpr int P2_NSL = 12;    // smem node slots
 constexpr u32 P2_NONE = 0xFFFFFFFFu;
 enum : u32 { P2_WB = 1, P2_SEND = 2, P2_END = 3, P2_STOP = 4 };
@@ -36,6 +37,7 @@ struct P2Ctl {
   u32 rq_head, rq_done;
   u32 rq[P2_RQ][4];
   u32 place_done;           // H2: placements completed
+  u32 fq[P2_H2D][7];        // H2: in-flight requests (type, a, b, c, smem source, min, max)
   u32 b[8];                 // thread-0 broadcasts
 };
 constexpr size_t P2CTL_BYTES = (sizeof(P2Ctl) + 127) / 128 * 128;
@@ -189,34 +191,68 @@ struct Pipe2 {
   // H2: sends and write-backs, in request order
   // ======================================================================================
   __device__ void h2_loop() {
-    u32 seen = 0, nplaced = 0;
+    // Requests are issued in order and completed in order with up to P2_H2D bulk groups in
+    // flight (one commit group per request): a send's flag (release) and a write-back's
+    // metadata are published only after cp.async.bulk.wait_group has retired that request's
+    // own group, so every message's data is globally visible before its flag.
+    constexpr u32 D = P2_H2D;
+    u32 seen = 0, nplaced = 0, inflight = 0, head_i = 0;
     u32 cache_l = P2_NONE, cache_c = 0;
+    auto retire = [&](u32 keep) {  // complete the oldest requests until <= keep are in flight
+      while (inflight > keep) {
+        if (keep == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+        else if (inflight - 1 == 1) asm volatile("cp.async.bulk.wait_group 1;" ::: "memory");
+        else if (inflight - 1 == 2) asm volatile("cp.async.bulk.wait_group 2;" ::: "memory");
+        else asm volatile("cp.async.bulk.wait_group 3;" ::: "memory");
+        const u32* f = pc->fq[head_i % D];
+        const u32 type = f[0], a = f[1], b = f[2], c = f[3];
+        if (f[4] != P2_NONE) release(f[4]);  // the smem source was read
+        asm volatile("fence.proxy.async.global;" ::: "memory");
+        if (type == P2_WB) {
+          st_relaxed(&H.meta[a].kmin, f[5]);
+          st_relaxed(&H.meta[a].kmax, f[6]);
+          if (c) {
+            st_relaxed(&H.meta[a].state, ST_AVAIL);
+            st_rel_cta(&pc->place_done, ++nplaced);
+          }
+        } else {  // SEND / END: header, then the flag (release)
+          const u32 l = a >> 8, m = b, rs = m % PIPE_NL;
+          u32* hd = P.rhdr + ((size_t)l * PIPE_NL + rs) * 4;
+          if (type == P2_SEND) { st_relaxed(hd + 0, c); st_relaxed(hd + 1, 0u); }
+          else { st_relaxed(hd + 0, 0u); st_relaxed(hd + 1, 1u); }
+          st_release(P.rflag + (size_t)l * PIPE_NL + rs, m + 1);
+        }
+        ++head_i;
+        --inflight;
+        ++seen;
+        st_rel_cta(&pc->rq_done, seen);
+      }
+    };
+    u32 issued = 0;
     for (;;) {
-      while (vld(&pc->rq_head) == seen) __nanosleep(32);
+      while (vld(&pc->rq_head) == issued) {
+        if (inflight) retire(0);
+        else __nanosleep(32);
+      }
       (void)ld_acq_cta(&pc->rq_head);
-      const u32* e = pc->rq[seen % P2_RQ];
+      const u32* e = pc->rq[issued % P2_RQ];
       const u32 type = e[0], a = e[1], b = e[2], c = e[3];
       if (type == P2_STOP) {
-        st_rel_cta(&pc->rq_done, seen + 1u);
+        retire(0);
+        ++issued;
+        ++seen;
+        st_rel_cta(&pc->rq_done, seen);
         return;
       }
+      retire(D - 1);  // room for one more group
+      u32* f = pc->fq[(head_i + inflight) % D];
+      f[0] = type; f[1] = a; f[2] = b; f[3] = c; f[4] = P2_NONE;
       if (type == P2_WB) {  // node a <- slot b (K entries); c = 1: placement (state AVAIL)
-        const u32 kmn = BK(b)[0], kmx = BK(b)[K - 1];
+        f[5] = BK(b)[0]; f[6] = BK(b)[K - 1]; f[4] = b;
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
         bulk_s2g(H.gk + (size_t)a * K, BK(b), NB);
         if (V) bulk_s2g(H.gv + (size_t)a * K, BV(b), NB);
-        asm volatile("cp.async.bulk.commit_group;" ::: "memory");
-        asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
-        release(b);
-        asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
-        asm volatile("fence.proxy.async.global;" ::: "memory");
-        st_relaxed(&H.meta[a].kmin, kmn);
-        st_relaxed(&H.meta[a].kmax, kmx);
-        if (c) {
-          st_relaxed(&H.meta[a].state, ST_AVAIL);
-          st_rel_cta(&pc->place_done, ++nplaced);
-        }
-      } else {  // P2_SEND (a = level, b = message, c = tar, slot in e[...]) / P2_END
+      } else {  // P2_SEND (a = level << 8 | slot, b = message, c = tar) / P2_END
         const u32 l = a >> 8, m = b;
         const u32 rs = m % PIPE_NL;
         if (m >= PIPE_NL) {  // flow control: the receiver consumed the slot's previous message
@@ -226,27 +262,17 @@ struct Pipe2 {
             if (cache_c < m + 1 - PIPE_NL) __nanosleep(64);
           }
         }
-        u32* hd = P.rhdr + ((size_t)l * PIPE_NL + rs) * 4;
         if (type == P2_SEND) {
           const u32 s = a & 0xFFu;
+          f[4] = s;
           asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
           bulk_s2g(ringk(l, rs), BK(s), NB);
           if (V) bulk_s2g(ringv(l, rs), BV(s), NB);
-          asm volatile("cp.async.bulk.commit_group;" ::: "memory");
-          asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
-          release(s);
-          asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
-          asm volatile("fence.proxy.async.global;" ::: "memory");
-          st_relaxed(hd + 0, c);
-          st_relaxed(hd + 1, 0u);
-        } else {
-          st_relaxed(hd + 0, 0u);
-          st_relaxed(hd + 1, 1u);
         }
-        st_release(P.rflag + (size_t)l * PIPE_NL + rs, m + 1);
       }
-      ++seen;
-      st_rel_cta(&pc->rq_done, seen);
+      asm volatile("cp.async.bulk.commit_group;" ::: "memory");  // (empty for END: retires in order)
+      ++inflight;
+      ++issued;
     }
   }
   __device__ __forceinline__ void send(u32 l, u32 m, u32 tar, u32 s) { h2(P2_SEND, (l << 8) | s, m, tar); }
