@@ -25,7 +25,7 @@ namespace bgpqd {
 constexpr u32 P2_PIN = 4;     // in-ring entries (H1 -> compute)
 constexpr u32 P2_RQ = 16;     // H2 request ring
 constexpr u32 P2_H2D = 4;     // H2 requests in flight (bulk groups)
-constexpr int P2_NSL = 12;    // smem node slots
+constexpr int P2_NSL = 24;    // smem node slots
 constexpr u32 P2_NONE = 0xFFFFFFFFu;
 enum : u32 { P2_WB = 1, P2_SEND = 2, P2_END = 3, P2_STOP = 4 };
 
@@ -105,9 +105,12 @@ struct Pipe2 {
     if (threadIdx.x == 0) { release(z); release(w); }
   }
   // compute threads: wait for in-ring entry m, read it, hand the entry back to H1
+  ull twait = 0;  // debug 128: cycles thread 0 waited for the next message (per stage)
   __device__ __forceinline__ void take(u32 m, u32& tar, u32& end, u32& is, u32& ns) {
     const u32 e = m % P2_PIN;
+    const ull t0 = (threadIdx.x == 0 && (C.debug & 128u)) ? clock64() : 0ull;
     mbar_wait(&pc->ibar[e], (m / P2_PIN) & 1u);
+    if (threadIdx.x == 0 && (C.debug & 128u)) twait += clock64() - t0;
     tar = pc->ent[e][0]; end = pc->ent[e][1]; is = pc->ent[e][2]; ns = pc->ent[e][3];
     cta_bar<NT>();
     if (threadIdx.x == 0) st_rel_cta(&pc->icons, m + 1u);
@@ -117,7 +120,7 @@ struct Pipe2 {
   // H1 of a level stage l (l >= 1): prefetch messages m = 0, 1, ... from ring l
   // ======================================================================================
   __device__ void h1_level(u32 l) {
-    u32 last_a = 0, nplace = 0;
+    u32 last_a = 0, nplace = 0, last_cons = 0;
     for (u32 m = 0;; ++m) {
       const u32 e = m % P2_PIN;
       while (m - vld(&pc->icons) >= P2_PIN) __nanosleep(32);
@@ -127,9 +130,10 @@ struct Pipe2 {
       while (ld_acquire(f) != m + 1) __nanosleep(32);
       const u32* hd = P.rhdr + ((size_t)l * PIPE_NL + slot) * 4;
       const u32 tar = ld_relaxed(hd + 0), end = ld_relaxed(hd + 1);
-      if (m > 0) {  // message m-1 has landed long ago: its ring slot may be reused
-        mbar_wait(&pc->ibar[(m - 1) % P2_PIN], ((m - 1) / P2_PIN) & 1u);
-        st_release(cons(l), m);
+      {  // ring slots of the messages the compute threads consumed (their loads landed) may be
+         // reused — no wait on the previous message's TMA, which would serialise its latency
+        const u32 done = vld(&pc->icons);
+        if (done != last_cons) { st_release(cons(l), done); last_cons = done; }
       }
       pc->ent[e][0] = tar; pc->ent[e][1] = end; pc->ent[e][2] = P2_NONE; pc->ent[e][3] = P2_NONE;
       if (end) {
@@ -168,22 +172,33 @@ struct Pipe2 {
 
   // H1 of the root stage: prefetch sorted batches j = 0, 1, ...
   __device__ void h1_root() {
+    u32 last_cons = 0;
+    const bool tm = (C.debug & 128u) != 0;
+    ull w_icons = 0, w_ready = 0, w_alloc = 0;
     for (u32 j = 0; j < (u32)C.n_ops; ++j) {
       const u32 e = j % P2_PIN;
+      ull t0 = tm ? clock64() : 0;
       while (j - vld(&pc->icons) >= P2_PIN) __nanosleep(32);
       (void)ld_acq_cta(&pc->icons);
+      if (tm) { const ull t = clock64(); w_icons += t - t0; t0 = t; }
       const u32 slot = j % PIPE_NSB;
       while (ld_acquire(P.sready + slot) != j + 1) __nanosleep(32);
-      if (j > 0) {
-        mbar_wait(&pc->ibar[(j - 1) % P2_PIN], ((j - 1) / P2_PIN) & 1u);
-        st_release(P.ctl + PC_ROOTCONS, j);  // the sorter may reuse batch j-1's slot
+      if (tm) { const ull t = clock64(); w_ready += t - t0; t0 = t; }
+      {  // the sorters may reuse the slots of the batches the root consumed (loads landed)
+        const u32 done = vld(&pc->icons);
+        if (done != last_cons) { st_release(P.ctl + PC_ROOTCONS, done); last_cons = done; }
       }
       const u32 is = alloc();
+      if (tm) { const ull t = clock64(); w_alloc += t - t0; t0 = t; }
       pc->ent[e][0] = op_size(j); pc->ent[e][1] = 0; pc->ent[e][2] = is; pc->ent[e][3] = P2_NONE;
       fence_proxy_async();
       mbar_arrive_expect_tx(&pc->ibar[e], V ? 2u * NB : NB);
       bulk_g2s(BK(is), P.sbk + (size_t)slot * K, NB, &pc->ibar[e]);
       if (V) bulk_g2s(BV(is), P.sbv + (size_t)slot * K, NB, &pc->ibar[e]);
+    }
+    if (tm) {
+      ull* tms = reinterpret_cast<ull*>(H.hdr + H_TIME);
+      atomicAdd(tms + 29, w_icons); atomicAdd(tms + 30, w_ready); atomicAdd(tms + 31, w_alloc);
     }
   }
 
@@ -244,7 +259,7 @@ struct Pipe2 {
         st_rel_cta(&pc->rq_done, seen);
         return;
       }
-      retire(D - 1);  // room for one more group
+      retire((C.debug & 4096u) ? 0u : D - 1);  // room for one more group (debug 4096: one at a time)
       u32* f = pc->fq[(head_i + inflight) % D];
       f[0] = type; f[1] = a; f[2] = b; f[3] = c; f[4] = P2_NONE;
       if (type == P2_WB) {  // node a <- slot b (K entries); c = 1: placement (state AVAIL)
@@ -496,8 +511,14 @@ __global__ void __launch_bounds__(NT + 64, 1) bgpq_ins_pipe2_kernel(HeapArgs H, 
     if (threadIdx.x == NT + 32) p.h2_loop();
     return;
   }
+  const ull t0 = clock64();
   if (b == 0) p.root_stage();
   else p.level_stage(b);
+  if (threadIdx.x == 0 && (C.debug & 128u) && b < 16) {
+    ull* tms = reinterpret_cast<ull*>(H.hdr + H_TIME);
+    atomicAdd(tms + b, p.twait);
+    atomicAdd(tms + 16 + b, clock64() - t0);
+  }
   if (threadIdx.x == 0) {
     ull* stat = reinterpret_cast<ull*>(H.hdr + H_STAT);
     for (int i = 0; i < NSTAT; ++i)

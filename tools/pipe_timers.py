@@ -1,19 +1,22 @@
-"""Per-level INSERT pipeline timers: python tools/pipe_timers.py [lg]"""
+"""Per-stage take-wait of the INSERT level pipeline: python tools/pipe_timers.py [lg]"""
 import sys, numpy as np, torch
 sys.path.insert(0, ".")
 import synth, paper_conf_icpp_chenhjz21_b200 as pkg
-pkg.set_debug(128)
 lg = int(sys.argv[1]) if len(sys.argv) > 1 else 27
 n = 1 << lg
 keys = synth.keys(n, seed=2)
 q = pkg.BGPQ(capacity=n, K=1024, values=False)
 dk = torch.from_numpy(keys.view(np.int32)).cuda()
+out = torch.empty(n, dtype=torch.int32, device="cuda")
+q.insert(dk); q.deletemin(n, out); torch.cuda.synchronize()   # reused-heap state, like the bench
+pkg.set_debug(128)
+t0 = q.timers().astype(np.float64)
 e = [torch.cuda.Event(enable_timing=True) for _ in range(2)]
 e[0].record(); q.insert(dk); e[1].record(); torch.cuda.synchronize()
-o = np.zeros(32, np.uint64); o[:] = q.timers()
-print("insert ms %.1f  (cycles, Mcyc)" % e[0].elapsed_time(e[1]))
-levels = list(range(1, 10)) + [14, 15, 16]
-for idx, l in enumerate(levels):
-    k = 3 * l if l < 10 else 3 * (l - 4)
-    if k + 2 < 32:
-        print("level %2d: take-wait %7.1f  merge %7.1f  total %7.1f" % (l, o[k] / 1e6, o[k + 1] / 1e6, o[k + 2] / 1e6))
+pkg.set_debug(0)
+d = q.timers().astype(np.float64) - t0
+ops = n // 1024
+print("insert ms %.1f   (cycles per op)" % e[0].elapsed_time(e[1]))
+for l in range(16):
+    print("stage %2d: take-wait %7.0f  total %7.0f" % (l, d[l] / ops, d[16 + l] / ops))
+print("root H1 (minus the stage 13-15 totals): wait icons %.0f  wait sorted batch %.0f  wait slot %.0f" % ((d[29]-d[16]) / ops, (d[30]-d[16]) / ops, (d[31]-d[16]) / ops))
