@@ -35,6 +35,7 @@ def main():
     ap.add_argument("--steps", type=int, default=3)
     ap.add_argument("--warmup", type=int, default=1)
     ap.add_argument("--budget", type=int, default=64, help="DELETEMINs per CTA per round (N > 1)")
+    ap.add_argument("--ctas", type=int, default=0, help="CTAs of the application kernel (0: all co-resident)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     args = ap.parse_args()
 
@@ -54,13 +55,14 @@ def main():
 
     if args.app == "knapsack":
         w, p, C = synth.knapsack_items(args.n_items, synth.SEEDS["C4"])
-        make = lambda: apps.KnapsackSearch(w, p, C, K=args.K, capacity=1 << 29)
+        make = lambda: apps.KnapsackSearch(w, p, C, K=args.K, capacity=1 << 29, ctas=args.ctas)
         workload = f"C4 knapsack B&B, {args.n_items} strongly correlated items, C={C}, K={args.K}"
     else:
         N = args.grid
         grid = synth.grid(N, N, args.rate, synth.SEEDS["C5"])
         dgrid = torch.from_numpy(grid).cuda()
-        make = lambda: apps.AStarSearch(None, (0, 0), (N - 1, N - 1), K=args.K, capacity=1 << 30, dgrid=dgrid)
+        make = lambda: apps.AStarSearch(None, (0, 0), (N - 1, N - 1), K=args.K, capacity=1 << 30, dgrid=dgrid,
+                                        ctas=args.ctas)
         workload = f"C5 A* {N}x{N} grid, {int(args.rate * 100)}% obstacles, K={args.K}"
 
     times, result, st_sum = [], None, None
@@ -93,6 +95,7 @@ def main():
                 "warmup": args.warmup, "times_s": times, "optimum": result[0], "rounds": result[1],
                 "bytes_moved_between_gpus": result[2], "dtype": "u32", "data": "synthetic",
                 "config": {"workload": workload, "budget_per_round": args.budget if world > 1 else None,
+                           "app_ctas": args.ctas or "all co-resident",
                            "parallelism": f"one BGPQ per GPU x{world}, NCCL incumbent all-reduce + rebalancing"},
                 "counters_per_solve": {k: v // args.steps for k, v in st_sum.items()}}
         if not args.no_cpu_baseline:

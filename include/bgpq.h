@@ -36,7 +36,7 @@ typedef struct bgpq bgpq_t;
 
 enum {
   BGPQ_OK = 0,
-  BGPQ_EINVAL = -1, /* bad argument (K not in {64,128,256,512,1024}, NULL pointer, ...) */
+  BGPQ_EINVAL = -1, /* bad argument (K not a power of two in 64..4096, NULL pointer, ...) */
   BGPQ_ENOMEM = -2, /* device allocation failed                                          */
   BGPQ_EFULL = -3,  /* sticky: an INSERT needed a node beyond the capacity; op dropped   */
   BGPQ_ECUDA = -4   /* a CUDA runtime call or kernel launch failed                       */
@@ -63,8 +63,9 @@ enum {
  *    Alg.2+3) with per-node locks, a lock warp per CTA taking the next level's locks ahead. */
 
 /* Create an empty heap able to hold `capacity` keys with node capacity K (§3.1:
- * every non-root node holds K sorted keys; k > 1).  K must be one of 64, 128, 256, 512,
- * 1024.  Allocates ceil(capacity/K)+2 node slots of K entries in device memory of the
+ * every non-root node holds K sorted keys; k > 1).  K must be a power of two in 64..4096
+ * (4096: keys only — a node pair with values exceeds the 227 KB of shared memory of a CTA;
+ * the paper stopped at 1K for the same reason on its GPU).  Allocates ceil(capacity/K)+2 node slots of K entries in device memory of the
  * current device.  bgpq_create stores keys and values (flags = BGPQ_FLAG_VALUES). */
 bgpq_t* bgpq_create(uint64_t capacity, uint32_t K);
 bgpq_t* bgpq_create_ex(uint64_t capacity, uint32_t K, uint32_t flags);
@@ -145,6 +146,7 @@ typedef struct {
   uint32_t flags;
   int device;
   int sm_count;
+  int ctas;       /* CTAs requested with bgpq_set_grid (0: all co-resident) — app kernels honour it */
 } bgpq_view_t;
 int bgpq_view(bgpq_t* q, bgpq_view_t* out);
 

@@ -23,7 +23,7 @@ NVCC_ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 NVCC_FLAGS = [*NVCC_ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC"]
 BUILD_DIR = os.path.join(_HERE, "build")
 # one object per (K, values) kernel table + the host-side C ABI (compiled in parallel)
-KERNEL_UNITS = [(k, v) for k in (64, 128, 256, 512, 1024) for v in (0, 1)]
+KERNEL_UNITS = [(k, v) for k in (64, 128, 256, 512, 1024, 2048, 4096) for v in (0, 1)]
 
 BGPQ_OK, BGPQ_EINVAL, BGPQ_ENOMEM, BGPQ_EFULL, BGPQ_ECUDA = 0, -1, -2, -3, -4
 FLAG_VALUES, FLAG_SERIAL, FLAG_LOCKS = 1, 2, 4
@@ -32,7 +32,7 @@ ST_EMPTY, ST_AVAIL, ST_TARGET, ST_MARKED = 0, 1, 2, 3
 STAT_NAMES = ("ins_ops", "ins_heapify_ops", "ins_levels", "ins_noop", "ins_swap", "ins_merge",
               "del_ops", "del_refill_ops", "del_levels", "del_lr_merge", "del_lr_skip", "marked",
               "keys_out", "root_spins", "del_lr_nomove", "del_cy_swap")
-VALID_K = (64, 128, 256, 512, 1024)
+VALID_K = (64, 128, 256, 512, 1024, 2048, 4096)  # K = 4096 keys only (values do not fit 227 KB)
 
 
 def _sources():
@@ -194,8 +194,8 @@ class BGPQ:
         default: insert calls as a level pipeline, deletemin calls on a top CTA with walker
         CTAs, mixed calls with per-node locks; locks=True: per-node-lock execution for every
         call."""
-        if K not in VALID_K:
-            raise ValueError(f"K must be one of {VALID_K}")
+        if K not in VALID_K or (K == 4096 and values):
+            raise ValueError(f"K must be one of {VALID_K} (4096: keys only)")
         flags = ((FLAG_VALUES if values else 0) | (FLAG_SERIAL if serial else 0)
                  | (FLAG_LOCKS if locks else 0))
         self._h = lib().bgpq_create_ex(int(capacity), int(K), flags)

@@ -46,10 +46,12 @@ class _Search:
     """Common part: one heap (values on), the 8-word state, pop / push of raw entries."""
     maximize = True
 
-    def __init__(self, K: int, capacity: int):
+    def __init__(self, K: int, capacity: int, ctas: int = 0):
         import torch
         self.K = K
         self.q = BGPQ(capacity=capacity, K=K, values=True)
+        if ctas:
+            self.q.set_grid(ctas)  # CTAs of the application kernel (0: all co-resident)
         self.state = torch.zeros(8, dtype=torch.int64, device="cuda")
         self._one_k = torch.zeros(1, dtype=torch.int32, device="cuda")
         self._one_v = torch.zeros(1, dtype=torch.int32, device="cuda")
@@ -87,9 +89,9 @@ class KnapsackSearch(_Search):
     """0-1 knapsack branch and bound (R23) on the current GPU."""
     maximize = True
 
-    def __init__(self, w: np.ndarray, p: np.ndarray, C: int, K: int = 1024, capacity: int = 1 << 27):
+    def __init__(self, w: np.ndarray, p: np.ndarray, C: int, K: int = 1024, capacity: int = 1 << 27, ctas: int = 0):
         import torch
-        super().__init__(K, capacity)
+        super().__init__(K, capacity, ctas)
         n = len(w)
         self.n, self.C = n, int(C)
         dw = torch.from_numpy(np.ascontiguousarray(w, np.uint32).view(np.int32)).cuda()
@@ -117,9 +119,10 @@ class AStarSearch(_Search):
     maximize = False
     INF = 0xFFFFFFFF
 
-    def __init__(self, grid: np.ndarray, start, target, K: int = 1024, capacity: int = 1 << 27, dgrid=None):
+    def __init__(self, grid: np.ndarray, start, target, K: int = 1024, capacity: int = 1 << 27, dgrid=None,
+                 ctas: int = 0):
         import torch
-        super().__init__(K, capacity)
+        super().__init__(K, capacity, ctas)
         N, M = grid.shape if dgrid is None else dgrid.shape
         self.N, self.M = int(N), int(M)
         self.start, self.target = tuple(start), tuple(target)

@@ -74,6 +74,8 @@ const KTable* ktab(u32 K, bool V) {
     case 256: return V ? &ktab_256_v() : &ktab_256_k();
     case 512: return V ? &ktab_512_v() : &ktab_512_k();
     case 1024: return V ? &ktab_1024_v() : &ktab_1024_k();
+    case 2048: return V ? &ktab_2048_v() : &ktab_2048_k();
+    case 4096: return V ? &ktab_4096_v() : &ktab_4096_k();
     default: return nullptr;
   }
 }
@@ -84,7 +86,7 @@ cudaError_t counted(cudaError_t e) {
   return e;
 }
 
-bool valid_K(u32 K) { return K == 64 || K == 128 || K == 256 || K == 512 || K == 1024; }
+bool valid_K(u32 K) { return K >= 64 && K <= 4096 && (K & (K - 1)) == 0; }
 
 HeapArgs heap_args(const bgpq* q) {
   HeapArgs H;
@@ -111,6 +113,7 @@ u32 depth_host(u32 i) {
 
 // Insert-only calls in the default execution run as a level pipeline (bgpq_pipe2.cuh).
 bool pipe_mode(const bgpq* q) { return !(q->flags & (BGPQ_FLAG_SERIAL | BGPQ_FLAG_LOCKS)); }
+bool has_pipe(const bgpq* q) { return ktab(q)->pipe_launch != nullptr; }
 
 // Allocates the pipeline rings and checks that its grid (one CTA per SM: root stage, one stage
 // per heap depth, sorters) is co-resident.  Returns BGPQ_OK, BGPQ_ENOMEM (allocation),
@@ -150,6 +153,7 @@ int ensure_pipe(bgpq* q) {
 // Deletemin-only calls in the default execution: top CTA + walkers (bgpq_dtop.cuh).
 // Debug bit 16 routes them to the per-node-lock execution instead (A/B comparisons).
 bool dt_mode(const bgpq* q) { return pipe_mode(q) && !(g_debug & 16u); }
+bool has_dt(const bgpq* q) { return ktab(q)->dt_launch != nullptr; }
 
 // Walker task list: one entry per hand-off (at most one per refill node, <= cap_nodes) plus
 // one ticket per walker CTA past the final count (each walker takes tickets until it sees
@@ -160,7 +164,7 @@ int ensure_dt(bgpq* q) {
   if (q->dt_ok) return BGPQ_OK;
   const bool V = (q->flags & BGPQ_FLAG_VALUES) != 0;
   int occ = 0;
-  if (ktab(q)->dt_prepare(&occ) != cudaSuccess || occ < 1) return fail(BGPQ_ECUDA);
+  if (has_dt(q) && (ktab(q)->dt_prepare(&occ) != cudaSuccess || occ < 1)) return fail(BGPQ_ECUDA);
   DtArgs& D = q->dt;
   const size_t n = dt_tasks(q);
   bool ok = cudaMalloc(&D.task_node, n * sizeof(u32)) == cudaSuccess;
@@ -192,6 +196,7 @@ bool ds_usable(bgpq* q, const CallArgs& C) {
   if ((reinterpret_cast<uintptr_t>(C.out_k) & 15u) || (C.out_v && (reinterpret_cast<uintptr_t>(C.out_v) & 15u)))
     return false;
   if (C.n < (u64)q->K) return false;
+  if (!ktab(q)->ds_launch) return false;
   if (q->ds_clusters < 0) {
     int cl = 0;
     if (ktab(q)->ds_prepare(q->sm_count, &cl) != cudaSuccess) {
@@ -228,6 +233,14 @@ int run_call(bgpq* q, const CallArgs& C, cudaStream_t s) {
       if (counted(ktab(q)->ds_launch(q->ds_clusters * DS_CL, heap_args(q), C, D, s)) != cudaSuccess)
         return fail(BGPQ_ECUDA);
     }
+    if (!has_dt(q)) {  // K >= 2048: the rest of the call on the per-node-lock engine
+      CallArgs C2 = C;
+      C2.op_base = D.op_base;
+      if (cudaMemsetAsync(q->hdr + H_CALL, 0, 2 * sizeof(u32), s) != cudaSuccess) return fail(BGPQ_ECUDA);
+      if (counted(ktab(q)->locks_launch(grid_for(q, C.n_ops), heap_args(q), C2, s)) != cudaSuccess)
+        return fail(BGPQ_ECUDA);
+      return BGPQ_OK;
+    }
     if (int rc = dt_epoch(q, s)) return rc;
     const u64* base = D.op_base;
     D = q->dt;
@@ -235,7 +248,7 @@ int run_call(bgpq* q, const CallArgs& C, cudaStream_t s) {
     if (counted(ktab(q)->dt_launch(q->sm_count, heap_args(q), C, D, s)) != cudaSuccess) return fail(BGPQ_ECUDA);
     return BGPQ_OK;
   }
-  if (C.mode == MODE_INSERT && pipe_mode(q)) {
+  if (C.mode == MODE_INSERT && pipe_mode(q) && has_pipe(q)) {
     if (int rc = ensure_pipe(q)) return rc;
     const PipeArgs& P = q->pipe;
     bool ok = cudaMemsetAsync(P.ctl, 0, PC_WORDS * sizeof(u32), s) == cudaSuccess;
@@ -280,7 +293,12 @@ bgpq_t* bgpq_create_ex(uint64_t capacity, uint32_t K, uint32_t flags) {
     return nullptr;
   }
   const bool V = (flags & BGPQ_FLAG_VALUES) != 0;
-  if (ktab(K, V)->locks_prepare(&q->occ) != cudaSuccess || q->occ < 1) {
+  if (!ktab(K, V)->locks_prepare || ktab(K, V)->locks_prepare(&q->occ) != cudaSuccess || q->occ < 1) {
+    if (!ktab(K, V)->locks_prepare) {  // (K, values) combination that no execution fits
+      delete q;
+      fail(BGPQ_EINVAL);
+      return nullptr;
+    }
     delete q;
     fail(BGPQ_ECUDA);
     return nullptr;
@@ -506,6 +524,7 @@ int bgpq_view(bgpq_t* q, bgpq_view_t* out) {
   out->flags = q->flags;
   out->device = q->device;
   out->sm_count = q->sm_count;
+  out->ctas = q->grid_req;
   return BGPQ_OK;
 }
 

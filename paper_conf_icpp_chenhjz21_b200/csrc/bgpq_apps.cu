@@ -406,6 +406,7 @@ int launch_app(bgpq_t* q, Kern kern, size_t q_smem, cudaStream_t s, int* grid_ou
   if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, ANT + 32, smem) != cudaSuccess || occ < 1)
     return BGPQ_ECUDA;
   *grid_out = v.sm_count * occ;
+  if (v.ctas > 0 && v.ctas < *grid_out) *grid_out = v.ctas;  // bgpq_set_grid
   return BGPQ_OK;
 }
 

@@ -13,6 +13,7 @@ namespace bgpqd {
 
 constexpr int NT = 512;  // compute threads per CTA (the paper's block size)
 
+// Entries are nullptr where an execution does not fit the shared memory at (K, V).
 struct KTable {
   // per-node-lock execution (bgpq_locks.cuh): prepare sets the smem attribute and returns
   // co-resident CTAs per SM in *occ
@@ -40,4 +41,6 @@ BGPQ_KTAB_DECL(128)
 BGPQ_KTAB_DECL(256)
 BGPQ_KTAB_DECL(512)
 BGPQ_KTAB_DECL(1024)
+BGPQ_KTAB_DECL(2048)
+BGPQ_KTAB_DECL(4096)
 #undef BGPQ_KTAB_DECL

@@ -908,6 +908,13 @@ __device__ __forceinline__ void lock_warp(OpL<K, V, NT>& op) {
 template <int K, bool V, int NT>
 __global__ void __launch_bounds__(NT + 32, 1) bgpq_locks_kernel(HeapArgs H, CallArgs C) {
   extern __shared__ __align__(128) unsigned char smem_raw[];
+  if (C.op_base) {  // the cluster engine executed the first ops of this deletemin call
+    const u64 b = *reinterpret_cast<volatile const u64*>(C.op_base);
+    C.n -= b * (u64)K;
+    C.n_ops -= b;
+    C.out_k += b * (u64)K;
+    if (C.out_v) C.out_v += b * (u64)K;
+  }
   LCtl* ctl = reinterpret_cast<LCtl*>(smem_raw);
   OpL<K, V, NT> op;
   op.H = H;

@@ -25,7 +25,12 @@ namespace bgpqd {
 constexpr u32 P2_PIN = 4;     // in-ring entries (H1 -> compute)
 constexpr u32 P2_RQ = 16;     // H2 request ring
 constexpr u32 P2_H2D = 4;     // H2 requests in flight (bulk groups)
-constexpr int P2_NSL = 24;    // smem node slots
+// smem node slots per stage: 24, fewer for the largest nodes (the stage needs >= 12: root,
+// pBuffer, the in-ring entries' item and node slots, the sends in flight)
+template <int K, bool V>
+__host__ __device__ constexpr int p2_nsl() {
+  return (size_t)24 * K * 4 * (V ? 2 : 1) <= 200704 ? 24 : 12;
+}
 constexpr u32 P2_NONE = 0xFFFFFFFFu;
 enum : u32 { P2_WB = 1, P2_SEND = 2, P2_END = 3, P2_STOP = 4 };
 
@@ -44,7 +49,7 @@ constexpr size_t P2CTL_BYTES = (sizeof(P2Ctl) + 127) / 128 * 128;
 
 template <int K, bool V>
 constexpr size_t pipe2_smem_bytes() {
-  return LCTL_BYTES + P2CTL_BYTES + (size_t)P2_NSL * K * 4 * (V ? 2 : 1);
+  return LCTL_BYTES + P2CTL_BYTES + (size_t)p2_nsl<K, V>() * K * 4 * (V ? 2 : 1);
 }
 
 __device__ __forceinline__ u32 vld(const u32* p) { return *reinterpret_cast<const volatile u32*>(p); }
@@ -483,7 +488,7 @@ __global__ void __launch_bounds__(NT + 64, 1) bgpq_ins_pipe2_kernel(HeapArgs H, 
     Pipe<K, V, NT> p;
     p.H = H; p.P = P; p.C = C; p.ctl = ctl;
     p.sk = reinterpret_cast<u32*>(smem_raw + LCTL_BYTES + P2CTL_BYTES);
-    p.sv = p.sk + P2_NSL * K;
+    p.sv = p.sk + p2_nsl<K, V>() * K;
     p.ph0 = 0; p.ph1 = 0;
     if (threadIdx.x == 0) {
       mbar_init(&ctl->bar, 1);
@@ -496,12 +501,12 @@ __global__ void __launch_bounds__(NT + 64, 1) bgpq_ins_pipe2_kernel(HeapArgs H, 
   Pipe2<K, V, NT> p;
   p.H = H; p.P = P; p.C = C; p.ctl = ctl; p.pc = pc;
   p.sk = reinterpret_cast<u32*>(smem_raw + LCTL_BYTES + P2CTL_BYTES);
-  p.sv = p.sk + P2_NSL * K;
+  p.sv = p.sk + p2_nsl<K, V>() * K;
   if (threadIdx.x == 0) {
     mbar_init(&ctl->bar, 1);
     for (u32 i = 0; i < P2_PIN; ++i) mbar_init(&pc->ibar[i], 1);
     for (int i = 0; i < NSTAT; ++i) ctl->st[i] = 0;
-    pc->pool = (1u << P2_NSL) - 1u;
+    pc->pool = (1u << p2_nsl<K, V>()) - 1u;
     pc->icons = 0; pc->rq_head = 0; pc->rq_done = 0; pc->place_done = 0;
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }

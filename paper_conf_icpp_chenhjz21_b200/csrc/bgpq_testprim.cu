@@ -46,8 +46,10 @@ __global__ void __launch_bounds__(TP_NT, 1)
   if (variant == 0) {  // the locks / pipeline SORT_SPLIT (bitonic for full keys-only K >= 512)
     sort_split<K, TP_NT, V>(sz, vz, na, sw, vw, nb, ma, sx, vx, sy, vy);
   } else if (variant == 1 || variant == 2) {  // the top CTA's group split (DT_GT threads)
-    if (threadIdx.x < DT_GT)
-      grp_split<K, V>((int)threadIdx.x, sz, vz, na, sw, vw, nb, ma, sx, vx, sy, vy, variant == 2);
+    if constexpr (K <= 1024) {
+      if (threadIdx.x < DT_GT)
+        grp_split<K, V>((int)threadIdx.x, sz, vz, na, sw, vw, nb, ma, sx, vx, sy, vy, variant == 2);
+    }
   } else if (variant == 3) {  // Sort(items) of the first na entries of Z (result in X)
     if (threadIdx.x < TP_NT) {
       const bool scratch = cta_sort<K, TP_NT, V>(sz, vz, na, sx, vx);
@@ -97,6 +99,13 @@ extern "C" int bgpq_test_prim(int variant, uint32_t K, int values, const uint32_
     TP_CASE(256)
     TP_CASE(512)
     TP_CASE(1024)
+    case 2048:
+      if (variant == 1 || variant == 2) return BGPQ_EINVAL;  // the top CTA runs K <= 1024 only
+      return values ? run<2048, true>(variant, zk, zv, wk, wv, na, nb, ma, n_cases, xk, xv, yk, yv, s)
+                    : run<2048, false>(variant, zk, zv, wk, wv, na, nb, ma, n_cases, xk, xv, yk, yv, s);
+    case 4096:
+      if (variant == 1 || variant == 2 || values) return BGPQ_EINVAL;  // keys only at K = 4096
+      return run<4096, false>(variant, zk, zv, wk, wv, na, nb, ma, n_cases, xk, xv, yk, yv, s);
     default:
       return BGPQ_EINVAL;
   }

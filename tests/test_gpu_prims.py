@@ -97,6 +97,12 @@ def test_sort_split_grid(variant, K, values):
     _run_split(variant, K, values, _grid(K), seed=1000 + K + variant)
 
 
+@pytest.mark.parametrize("K,values", [(2048, False), (2048, True), (4096, False)])
+def test_sort_split_grid_large_k(K, values):
+    """K beyond the paper's 1K (NEXT-3): the lock / pipeline executions' SORT_SPLIT."""
+    _run_split(0, K, values, _grid(K), seed=3000 + K)
+
+
 @pytest.mark.parametrize("K", [512, 1024])
 @pytest.mark.parametrize("variant", [0, 1])
 def test_bitonic_split_full_random(variant, K):
@@ -107,8 +113,8 @@ def test_bitonic_split_full_random(variant, K):
     _run_split(variant, K, False, cases, seed=77 + K)
 
 
-@pytest.mark.parametrize("values", [False, True])
-@pytest.mark.parametrize("K", VALID_K)
+@pytest.mark.parametrize("K,values", [(k, v) for k in VALID_K for v in (False, True)] +
+                         [(2048, False), (2048, True), (4096, False)])
 def test_cta_sort(K, values):
     rng = np.random.default_rng(K)
     sizes = sorted(set([1, 2, 31, 32, 33, 63, 64, 65, K // 2, K - 1, K] + list(rng.integers(1, K + 1, 20))))
