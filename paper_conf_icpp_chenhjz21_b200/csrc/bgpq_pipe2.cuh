@@ -14,9 +14,13 @@
 //      level's ring slot, completion, proxy fence, release of the flag, with flow control)
 //      and node write-backs (bulk store + cached min/max + state for placements, Alg.1 l.9-10);
 // so the compute threads only take decisions and run SORT_SPLITs.  Path nodes of depth l are
-// non-decreasing in the message order (tar = heapSize + 1 grows), so a node is never reloaded
-// after the stage moved away from it; the one hazard — a node placed by this stage and needed
-// as a path node later in the same call — makes H1 wait for H2's completion of the placements.
+// non-decreasing in the message order while tar stays at one depth (tar = heapSize + 1
+// grows); two hazards remain: a node placed by this stage and needed as a path node later in
+// the same call (H1 waits for H2's completion of the placements), and the restart of the
+// path at the leftmost node of depth l when tar enters the next depth — that node was this
+// stage's path node before, so H1 waits until every earlier message was processed and its
+// write-back retired (a round-1 H1 could prefetch the stale HBM copy while the compute still
+// held the dirty one: keys lost on small reused heaps, seen at K = 4096).
 #pragma once
 #include "bgpq_pipe.cuh"
 
@@ -42,6 +46,7 @@ struct P2Ctl {
   u32 rq_head, rq_done;
   u32 rq[P2_RQ][4];
   u32 place_done;           // H2: placements completed
+  u32 mdone;                // compute: messages fully processed (their H2 requests issued)
   u32 fq[P2_H2D][7];        // H2: in-flight requests (type, a, b, c, smem source, min, max)
   u32 b[8];                 // thread-0 broadcasts
 };
@@ -135,8 +140,13 @@ struct Pipe2 {
       while (ld_acquire(f) != m + 1) __nanosleep(32);
       const u32* hd = P.rhdr + ((size_t)l * PIPE_NL + slot) * 4;
       const u32 tar = ld_relaxed(hd + 0), end = ld_relaxed(hd + 1);
-      {  // ring slots of the messages the compute threads consumed (their loads landed) may be
-         // reused — no wait on the previous message's TMA, which would serialise its latency
+      if (C.debug & 8192u) {  // test switch: the previous message's load landed, release it
+        if (m > 0) {
+          mbar_wait(&pc->ibar[(m - 1) % P2_PIN], ((m - 1) / P2_PIN) & 1u);
+          st_release(cons(l), m);
+        }
+      } else {  // ring slots of the messages the compute threads consumed (their loads landed)
+                // may be reused — no wait on the previous message's TMA
         const u32 done = vld(&pc->icons);
         if (done != last_cons) { st_release(cons(l), done); last_cons = done; }
       }
@@ -153,6 +163,14 @@ struct Pipe2 {
       if (dt > l) {
         a = tar >> (dt - l);
         if (a != last_a) {
+          if (a < last_a) {
+            // tar entered the next depth: the path at depth l restarts at the leftmost node,
+            // which this stage held (and may have written back) earlier in the call — load it
+            // only after every earlier message was processed and its write-back retired
+            while (ld_acq_cta(&pc->mdone) < m) __nanosleep(32);
+            const u32 h = ld_acq_cta(&pc->rq_head);
+            while ((int)(ld_acq_cta(&pc->rq_done) - h) < 0) __nanosleep(32);
+          }
           last_a = a;
           ns = alloc();
           bytes += V ? 2u * NB : NB;
@@ -431,7 +449,7 @@ struct Pipe2 {
       if (end) break;
       const u32 dt = depth_of(tar);
       if (dt == l) {  // l.9-10: Heap[tar] <- items (state AVAIL)
-        if (tid == 0) h2(P2_WB, tar, I, 1u);
+        if (tid == 0) { h2(P2_WB, tar, I, 1u); st_rel_cta(&pc->mdone, m + 1u); }
         continue;
       }
       if (ns != P2_NONE) {  // the path node of depth l changed: write the old one back
@@ -459,7 +477,7 @@ struct Pipe2 {
         dirty = 1;
         ++nmerge;
       }
-      if (tid == 0) send(l + 1, sent, tar, I);
+      if (tid == 0) { send(l + 1, sent, tar, I); st_rel_cta(&pc->mdone, m + 1u); }
       ++sent;
     }
     if (tid == 0) {
@@ -507,7 +525,7 @@ __global__ void __launch_bounds__(NT + 64, 1) bgpq_ins_pipe2_kernel(HeapArgs H, 
     for (u32 i = 0; i < P2_PIN; ++i) mbar_init(&pc->ibar[i], 1);
     for (int i = 0; i < NSTAT; ++i) ctl->st[i] = 0;
     pc->pool = (1u << p2_nsl<K, V>()) - 1u;
-    pc->icons = 0; pc->rq_head = 0; pc->rq_done = 0; pc->place_done = 0;
+    pc->icons = 0; pc->rq_head = 0; pc->rq_done = 0; pc->place_done = 0; pc->mdone = 0;
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();

@@ -373,3 +373,24 @@ def test_full_size_c2_properties(mode):
     assert np.all(out[1:] >= out[:-1])
     assert np.array_equal(out, srt)
     assert q.size() == 0
+
+
+@pytest.mark.parametrize("K", [64, 256, 1024, 4096])
+def test_pipelined_insert_reused_small_heap_layout(K):
+    """Regression: on a small heap refilled after drains, the level stages revisit the leftmost
+    path node of their depth each time tar enters a new depth; the stage's prefetch helper must
+    not load it before the compute's write-back of that node retired (keys were lost at K =
+    4096).  The layout after every insert call equals the sequential Alg.1 model's."""
+    n = 40 * K + 37
+    keys = synth.keys(n, seed=synth.SEEDS["C3"] + K)
+    q = pkg.BGPQ(capacity=n, K=K, values=False)
+    seq = oracle.SeqBGPQ(K, q.slots() - 1)
+    for rep in range(5):
+        q.insert(_dev(keys))
+        for off in range(0, n, K):
+            seq.insert(keys[off:min(off + K, n)])
+        _compare_layout(q, seq)
+        ok, _ = q.deletemin(n)
+        want = np.concatenate([seq.deletemin(K)[0] for _ in range((n + K - 1) // K)])
+        assert np.array_equal(_host(ok), want), rep
+    q.close()
