@@ -164,7 +164,8 @@ def _pin_one_core():
 def _config(args):
     w = 8 if args.values else 4
     ex = ({"insert": "level pipeline (bgpq_ins_pipe2_kernel: root stage, one stage CTA per heap depth, sorter CTAs)",
-           "deletemin": "top CTA + walker CTAs (bgpq_dtop_kernel)"} if args.mode == "default" else
+           "deletemin": ("cluster engine (bgpq_dsys_kernel: 5-CTA cluster over depths 0-4, walker CTAs "
+                         "below) + the call's tail on the top CTA (bgpq_dtop_kernel)")} if args.mode == "default" else
           {"insert": "per-node locks (bgpq_locks_kernel, FLAG_LOCKS)",
            "deletemin": "per-node locks (bgpq_locks_kernel, FLAG_LOCKS)"})
     return {"workload": (f"C2 phased: insert 2^{args.n_log2} {args.dist} uint32 keys into an empty BGPQ "
@@ -391,8 +392,8 @@ def main():
     ap.add_argument("--mix-log2", type=int, default=None, help="mix keys inserted (default: --n-log2)")
     ap.add_argument("--grid", type=int, default=0, help="mix: persistent CTAs of the mixed call (0 = all co-resident)")
     ap.add_argument("--mode", default="default", choices=["default", "locks"],
-                    help="execution: default (insert level pipeline + deletemin top CTA with walkers "
-                         "taking the paper's per-node locks), or the paper-literal per-node-lock engine "
+                    help="execution: default (insert level pipeline + deletemin cluster engine and top-CTA tail, "
+                         "walkers taking the paper's per-node locks below), or the paper-literal per-node-lock engine "
                          "for every call (BGPQ_FLAG_LOCKS)")
     args = ap.parse_args()
     if args.mix_log2 is None:
@@ -537,7 +538,8 @@ def main():
             "parallelism": "replicas only (one linearizable heap per GPU)",
             "phases_ms": {"insert": float(np.mean(ins_ms)), "deletemin": float(np.mean(del_ms))},
             "roofline": {"bound": "hbm",
-                         "kernel": ("bgpq_dtop_kernel (DELETEMIN launch)" if args.mode == "default"
+                         "kernel": ("bgpq_dsys_kernel (+ its bgpq_dtop_kernel tail, ~2% of the DELETEMIN call "
+                                    "in the ncu launch list profiles/r2/launches_r2.csv)" if args.mode == "default"
                                     else "bgpq_locks_kernel (DELETEMIN launch)"),
                          "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
                          "traffic": traffic, "traffic_source": traffic_src, "peak_source": peak_src,
