@@ -35,7 +35,8 @@ def main():
     ap.add_argument("--steps", type=int, default=3)
     ap.add_argument("--warmup", type=int, default=1)
     ap.add_argument("--budget", type=int, default=64, help="DELETEMINs per CTA per round (N > 1)")
-    ap.add_argument("--ctas", type=int, default=0, help="CTAs of the application kernel (0: all co-resident)")
+    ap.add_argument("--ctas", type=int, default=None,
+                    help="CTAs of the application kernel (0: all co-resident; default: the app's DEFAULT_CTAS)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     args = ap.parse_args()
 
@@ -95,7 +96,8 @@ def main():
                 "warmup": args.warmup, "times_s": times, "optimum": result[0], "rounds": result[1],
                 "bytes_moved_between_gpus": result[2], "dtype": "u32", "data": "synthetic",
                 "config": {"workload": workload, "budget_per_round": args.budget if world > 1 else None,
-                           "app_ctas": args.ctas or "all co-resident",
+                           "app_ctas": (args.ctas if args.ctas is not None else
+                                        (apps.KnapsackSearch if args.app == "knapsack" else apps.AStarSearch).DEFAULT_CTAS),
                            "parallelism": f"one BGPQ per GPU x{world}, NCCL incumbent all-reduce + rebalancing"},
                 "counters_per_solve": {k: v // args.steps for k, v in st_sum.items()}}
         if not args.no_cpu_baseline:

@@ -45,13 +45,18 @@ def _bind():
 class _Search:
     """Common part: one heap (values on), the 8-word state, pop / push of raw entries."""
     maximize = True
+    # CTAs of the application kernel when the caller does not choose (None); 0 = all
+    # co-resident.  From the one-B200 sweeps in profiles/r2 (ks_ctas_*.json, astar_ctas_*.json):
+    # fewer CTAs contend less for the root lock when the frontier is narrow.
+    DEFAULT_CTAS = 0
 
-    def __init__(self, K: int, capacity: int, ctas: int = 0):
+    def __init__(self, K: int, capacity: int, ctas: int | None = None):
         import torch
         self.K = K
         self.q = BGPQ(capacity=capacity, K=K, values=True)
+        ctas = self.DEFAULT_CTAS if ctas is None else ctas
         if ctas:
-            self.q.set_grid(ctas)  # CTAs of the application kernel (0: all co-resident)
+            self.q.set_grid(ctas)
         self.state = torch.zeros(8, dtype=torch.int64, device="cuda")
         self._one_k = torch.zeros(1, dtype=torch.int32, device="cuda")
         self._one_v = torch.zeros(1, dtype=torch.int32, device="cuda")
@@ -88,8 +93,10 @@ class _Search:
 class KnapsackSearch(_Search):
     """0-1 knapsack branch and bound (R23) on the current GPU."""
     maximize = True
+    DEFAULT_CTAS = 64  # C4: 1.50 s at 64 CTAs vs 1.79 s with all 148
 
-    def __init__(self, w: np.ndarray, p: np.ndarray, C: int, K: int = 1024, capacity: int = 1 << 27, ctas: int = 0):
+    def __init__(self, w: np.ndarray, p: np.ndarray, C: int, K: int = 1024, capacity: int = 1 << 27,
+                 ctas: int | None = None):
         import torch
         super().__init__(K, capacity, ctas)
         n = len(w)
@@ -118,9 +125,10 @@ class AStarSearch(_Search):
     """A* on an N x M obstacle grid (R24) on the current GPU."""
     maximize = False
     INF = 0xFFFFFFFF
+    DEFAULT_CTAS = 8  # C5 10 %: 2.06 s at 8 CTAs vs 3.64 s with all 148
 
     def __init__(self, grid: np.ndarray, start, target, K: int = 1024, capacity: int = 1 << 27, dgrid=None,
-                 ctas: int = 0):
+                 ctas: int | None = None):
         import torch
         super().__init__(K, capacity, ctas)
         N, M = grid.shape if dgrid is None else dgrid.shape
