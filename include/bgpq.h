@@ -155,7 +155,13 @@ int bgpq_view(bgpq_t* q, bgpq_view_t* out);
  *   8   accumulate thread-0 cycle timers in the header (read with bgpq_timers);
  *   16  run deletemin-only calls on the per-node-lock engine instead of the top CTA;
  *   64  register-window merge path instead of the warp-cooperative one on the top CTA;
- *   128 light top-CTA timers (plan / phase A / phase B).
+ *   128 light top-CTA timers (plan / phase A / phase B);
+ *   256 deletemin calls skip the cluster engine (top CTA / lock engine only);
+ *   1024 cluster-engine role timers and walker first-level timers;
+ *   32768 schedule forcing for tests: every INSERT on the per-node-lock engine holds its
+ *         target node (state TARGET) 20 us before the placement (Alg.1 l.8-13), so concurrent
+ *         DELETEMINs take the TARGET -> MARKED steal (Alg.2 l.7-9) and the one-AVAIL-
+ *         child path of the heapify (Alg.3 l.5-8).
  * bgpq_timers: copies the 32 uint64 cycle counters of the handle to out32 (host);
  * synchronizes the device. */
 int bgpq_set_debug(uint32_t bits);

@@ -92,6 +92,11 @@ struct OpL {
   static constexpr u32 NBYTES = K * 4u;
   HeapArgs H;
   bool timing;
+  // schedule forcing (test only, bgpq_set_debug bit 32768): an INSERT holds its target node in
+  // state TARGET this many ns before the placement (Alg.1 l.8-13), so concurrent DELETEMINs
+  // meet the in-flight insert: the refill steals it (TARGET -> MARKED, Alg.2 l.7-9) and
+  // heapify walks see exactly one AVAIL child (R5)
+  u32 delay_ns = 0;
   ull* tm;  // -> ctl->tm
   int tmerge = LT_DEL_MERGE, tstore = LT_DEL_STORE;  // timer ids of the current op type
   __device__ __forceinline__ ull now() const { return timing ? clock64() : 0ull; }
@@ -453,6 +458,7 @@ struct OpL {
     // ---- l.8: LOCK(tar); UNLOCK(PARENT(cur)); l.9-14
     cta_bar<NT>();
     if (tid == 0) {
+      for (u32 w = 0; w < delay_ns; w += 1000) __nanosleep(1000);  // test-only schedule forcing
       const ull tt = now();
       if (held == 1) wait_t_done();  // agent T's LOCK(tar) of l.5-6 must be over first
       lock_acquire(lk(tar));
@@ -925,6 +931,7 @@ __global__ void __launch_bounds__(NT + 32, 1) bgpq_locks_kernel(HeapArgs H, Call
   op.st = ctl->st;
   op.tm = ctl->tm;
   op.timing = (C.debug & 8u) != 0;
+  op.delay_ns = (C.debug & 32768u) ? 20000u : 0u;
   if (threadIdx.x == 0) {
     for (int i = 0; i < NSTAT; ++i) ctl->st[i] = 0;
     for (int i = 0; i < 32; ++i) ctl->tm[i] = 0;

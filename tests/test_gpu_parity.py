@@ -311,6 +311,36 @@ def test_marked_handoff_replay(mode):
         assert total_marked > 0
 
 
+def test_forced_collaboration_replay():
+    """Schedule forcing (bgpq_set_debug 32768): inserts hold their target node TARGET for 20 us
+    before the placement, so concurrent deletemins must steal from in-flight inserts
+    (TARGET -> MARKED, Alg.2 l.7-9; the insert then fills the root, Alg.1 l.11-13) and
+    walk past a TARGET child (exactly one AVAIL child, R5).  Both paths are asserted to fire
+    and the ticket-order replay stays bit-exact."""
+    K = 64
+    marked = skip = 0
+    pkg.set_debug(32768)
+    try:
+        for seed in range(2):
+            types, _ = synth.random_ops(2000, K, seed=80 + seed, p_insert=0.5)
+            sizes = np.full(len(types), K, np.uint32)
+            keys, in_off = _mixed_inputs(types, sizes, K, seed=90 + seed)
+            q = pkg.BGPQ(capacity=len(keys) + K, K=K, values=True, locks=True)
+            outk, outv, cnt, lin = _run_mixed(q, types, sizes, keys, in_off)
+            _replay_check(types, sizes, keys, in_off, outk, outv, cnt, lin)
+            for j in np.nonzero(types == 1)[0]:
+                assert np.array_equal(keys[outv[j, :cnt[j]]], outk[j, :cnt[j]])
+            assert _gpu_inv(q) == (0, 0)
+            st = q.stats()
+            marked += st["marked"]
+            skip += st["del_lr_skip"]
+            q.close()
+    finally:
+        pkg.set_debug(0)
+    print("forced: MARKED", marked, "one-AVAIL-child levels", skip)
+    assert marked > 0 and skip > 0
+
+
 # --------------------------------------------------------------------------------------
 # edge cases
 # --------------------------------------------------------------------------------------
