@@ -98,9 +98,14 @@ struct Pipe2 {
     if (s != P2_NONE) atomicOr(&pc->pool, 1u << s);
   }
   // ---- thread 0 -> H2
+  ull th2 = 0;  // debug 128|16384: cycles thread 0 waited for room in H2's request ring
   __device__ __forceinline__ void h2(u32 type, u32 a = 0, u32 b = 0, u32 c = 0) {
     const u32 h = pc->rq_head;
-    while (h - vld(&pc->rq_done) >= P2_RQ) __nanosleep(32);
+    if (h - vld(&pc->rq_done) >= P2_RQ) {
+      const ull t0 = (C.debug & 16384u) ? clock64() : 0ull;
+      while (h - vld(&pc->rq_done) >= P2_RQ) __nanosleep(32);
+      if (C.debug & 16384u) th2 += clock64() - t0;
+    }
     u32* e = pc->rq[h % P2_RQ];
     e[0] = type; e[1] = a; e[2] = b; e[3] = c;
     st_rel_cta(&pc->rq_head, h + 1u);
@@ -109,9 +114,11 @@ struct Pipe2 {
   __device__ __forceinline__ void merge2(u32 z, u32 na, u32 w, u32 nb, u32 ma, u32& x, u32& y) {
     if (threadIdx.x == 0) { ctl->b[20] = alloc(); ctl->b[21] = alloc(); }
     cta_bar<NT>();
+    const ull ts = (threadIdx.x == 0 && (C.debug & 131072u)) ? clock64() : 0ull;
     x = ctl->b[20]; y = ctl->b[21];
     sort_split<K, NT, V>(BK(z), BV(z), (int)na, BK(w), BV(w), (int)nb, (int)ma, BK(x), BV(x), BK(y), BV(y));
     cta_bar<NT>();
+    if (threadIdx.x == 0 && (C.debug & 131072u)) twait += clock64() - ts;  // debug 131072: split only
     if (threadIdx.x == 0) { release(z); release(w); }
   }
   // compute threads: wait for in-ring entry m, read it, hand the entry back to H1
@@ -120,7 +127,7 @@ struct Pipe2 {
     const u32 e = m % P2_PIN;
     const ull t0 = (threadIdx.x == 0 && (C.debug & 128u)) ? clock64() : 0ull;
     mbar_wait(&pc->ibar[e], (m / P2_PIN) & 1u);
-    if (threadIdx.x == 0 && (C.debug & 128u)) twait += clock64() - t0;
+    if (threadIdx.x == 0 && (C.debug & 128u) && !(C.debug & 65536u)) twait += clock64() - t0;
     tar = pc->ent[e][0]; end = pc->ent[e][1]; is = pc->ent[e][2]; ns = pc->ent[e][3];
     cta_bar<NT>();
     if (threadIdx.x == 0) st_rel_cta(&pc->icons, m + 1u);
@@ -443,6 +450,13 @@ struct Pipe2 {
     const int tid = threadIdx.x;
     u32 N = P2_NONE, cur = 0, dirty = 0, sent = 0;
     ull lv = 0, nnoop = 0, nswap = 0, nmerge = 0;
+    // two spare slots receive a merge's outputs and its inputs become the next spares: tracked
+    // identically by every compute thread, so a merge needs no slot-pool atomics and no
+    // barrier before the split (the inputs were last read before the previous split's barrier;
+    // neither input is ever referenced by a pending H2 request)
+    if (tid == 0) { ctl->b[22] = alloc(); ctl->b[23] = alloc(); }
+    cta_bar<NT>();
+    u32 sp0 = ctl->b[22], sp1 = ctl->b[23];
     for (u32 m = 0;; ++m) {
       u32 tar, end, I, ns;
       take(m, tar, end, I, ns);
@@ -471,8 +485,12 @@ struct Pipe2 {
         dirty = 1;
         ++nswap;
       } else {
-        u32 a, b;
-        merge2(N, K, I, K, K, a, b);
+        const ull tq = (tid == 0 && (C.debug & 65536u)) ? clock64() : 0ull;
+        sort_split<K, NT, V>(BK(N), BV(N), K, BK(I), BV(I), K, K, BK(sp0), BV(sp0), BK(sp1), BV(sp1));
+        cta_bar<NT>();
+        if (tid == 0 && (C.debug & 65536u)) twait += clock64() - tq;  // debug 65536: merge time instead
+        const u32 a = sp0, b = sp1;
+        sp0 = N; sp1 = I;
         N = a; I = b;
         dirty = 1;
         ++nmerge;
@@ -484,6 +502,8 @@ struct Pipe2 {
       if (l < P.depth) send_end(l + 1, sent);
       if (dirty) h2(P2_WB, cur, N, 0u);
       else release(N);
+      release(sp0);
+      release(sp1);
     }
     h2_drain();
     if (tid == 0) {
@@ -540,7 +560,7 @@ __global__ void __launch_bounds__(NT + 64, 1) bgpq_ins_pipe2_kernel(HeapArgs H, 
   if (threadIdx.x == 0 && (C.debug & 128u) && b < 16) {
     ull* tms = reinterpret_cast<ull*>(H.hdr + H_TIME);
     atomicAdd(tms + b, p.twait);
-    atomicAdd(tms + 16 + b, clock64() - t0);
+    atomicAdd(tms + 16 + b, (C.debug & 16384u) ? p.th2 : clock64() - t0);
   }
   if (threadIdx.x == 0) {
     ull* stat = reinterpret_cast<ull*>(H.hdr + H_STAT);
