@@ -57,6 +57,8 @@ struct Queue {
     H.meta = h.meta;
     H.hdr = h.hdr;
     H.cap = h.cap;
+    H.xk = nullptr;  // carried-keys sources are heap nodes here (no cluster-engine scratch)
+    H.xv = nullptr;
     bgpqd::LCtl* ctl = reinterpret_cast<bgpqd::LCtl*>(smem);
     op.H = H;
     op.ctl = ctl;

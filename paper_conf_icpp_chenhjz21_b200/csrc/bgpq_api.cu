@@ -60,6 +60,10 @@ struct bgpq {
   u64 stage_n = 0;
   int ds_clusters = -1;    // co-resident clusters of the cluster DELETEMIN engine (-1: not queried)
   u64* ds_base = nullptr;  // device: ops of the current deletemin call done by that engine
+  u32* xk = nullptr;       // mixed calls on the cluster engine: sorted INSERT batch per op pair
+  u32* xv = nullptr;
+  u64 x_pairs = 0;         // pairs xk / xv hold
+  u32* pair_end = nullptr; // device word: pairs of the current mixed call the engine may run
   bool attr_dt = false;    // kernel attributes set / occupancy checked on q->device
   bool attr_pipe = false;
 };
@@ -95,6 +99,8 @@ HeapArgs heap_args(const bgpq* q) {
   H.meta = q->meta;
   H.hdr = q->hdr;
   H.cap = q->cap_nodes;
+  H.xk = q->xk;
+  H.xv = (q->flags & BGPQ_FLAG_VALUES) ? q->xv : nullptr;
   return H;
 }
 
@@ -208,6 +214,37 @@ bool ds_usable(bgpq* q, const CallArgs& C) {
   return q->ds_clusters >= 8;  // the role cluster + >= 7 clusters of walkers
 }
 
+// Mixed calls whose op stream starts with (INSERT(K), DELETEMIN(K)) pairs (the utilisation
+// workload) run those pairs on the cluster engine (bgpq_dsys.cuh: ds_r0_mixed) and the
+// rest on the per-node-lock engine; debug bit 256 disables it like for deletemin calls.
+bool dsm_usable(bgpq* q, const CallArgs& C) {
+  if (!ktab(q)->ms_launch || C.n_ops < 2) return false;
+  CallArgs C1 = C;
+  C1.n = q->K;  // ds_usable's size test is about deletemin calls
+  return ds_usable(q, C1);
+}
+
+int ensure_mixed(bgpq* q, u64 pairs) {
+  if (!q->pair_end && cudaMalloc(&q->pair_end, sizeof(u32)) != cudaSuccess) {
+    cudaGetLastError();
+    return fail(BGPQ_ENOMEM);
+  }
+  if (q->x_pairs >= pairs) return BGPQ_OK;
+  cudaFree(q->xk);
+  cudaFree(q->xv);
+  q->xk = q->xv = nullptr;
+  q->x_pairs = 0;
+  const size_t bytes = pairs * (size_t)q->K * sizeof(u32);
+  bool ok = cudaMalloc(&q->xk, bytes) == cudaSuccess;
+  if (ok && (q->flags & BGPQ_FLAG_VALUES)) ok = cudaMalloc(&q->xv, bytes) == cudaSuccess;
+  if (!ok) {
+    cudaGetLastError();
+    return fail(BGPQ_ENOMEM);
+  }
+  q->x_pairs = pairs;
+  return BGPQ_OK;
+}
+
 int dt_epoch(bgpq* q, cudaStream_t s) {
   DtArgs& D = q->dt;
   D.epoch += 1;
@@ -256,6 +293,25 @@ int run_call(bgpq* q, const CallArgs& C, cudaStream_t s) {
     ok = ok && cudaMemsetAsync(P.rflag, 0, (size_t)PIPE_MAXL * PIPE_NL * sizeof(u32), s) == cudaSuccess;
     if (!ok) return fail(BGPQ_ECUDA);
     if (counted(ktab(q)->pipe_launch(q->pipe_grid, heap_args(q), P, C, s)) != cudaSuccess) return fail(BGPQ_ECUDA);
+    return BGPQ_OK;
+  }
+  if (C.mode == MODE_MIXED && dt_mode(q) && dsm_usable(q, C)) {
+    // leading op pairs: Sort(items) of every pair's INSERT, then the cluster engine; the
+    // per-node-lock engine continues at the first op the engine did not run (H_FETCH)
+    if (int rc = ensure_dt(q)) return rc;
+    if (int rc = ensure_mixed(q, C.n_ops / 2)) return rc;
+    if (cudaMemsetAsync(q->pair_end, 0xFF, sizeof(u32), s) != cudaSuccess) return fail(BGPQ_ECUDA);
+    CallArgs Cm = C;
+    Cm.pair_end = q->pair_end;
+    if (counted(ktab(q)->ms_launch(q->sm_count * 4, heap_args(q), Cm, s)) != cudaSuccess) return fail(BGPQ_ECUDA);
+    if (int rc = dt_epoch(q, s)) return rc;
+    DtArgs D = q->dt;
+    D.op_base = q->ds_base;
+    if (cudaMemsetAsync(q->hdr + H_CALL, 0, 2 * sizeof(u32), s) != cudaSuccess) return fail(BGPQ_ECUDA);
+    if (counted(ktab(q)->ds_launch(q->ds_clusters * DS_CL, heap_args(q), Cm, D, s)) != cudaSuccess)
+      return fail(BGPQ_ECUDA);
+    if (counted(ktab(q)->locks_launch(grid_for(q, C.n_ops), heap_args(q), C, s)) != cudaSuccess)
+      return fail(BGPQ_ECUDA);
     return BGPQ_OK;
   }
   // reset the per-call ticket and fetch counter (header words H_CALL, H_FETCH)
@@ -336,6 +392,9 @@ void bgpq_destroy(bgpq_t* q) {
   cudaFree(q->dt.task_seq);
   cudaFree(q->dt.task_go);
   cudaFree(q->ds_base);
+  cudaFree(q->xk);
+  cudaFree(q->xv);
+  cudaFree(q->pair_end);
   cudaFree(q->dt.ctl);
   PipeArgs& P = q->pipe;
   u32* pbufs[] = {P.ctl, P.sbk, P.sbv, P.sready, P.rk, P.rv, P.rhdr, P.rflag};

@@ -45,6 +45,8 @@ constexpr u32 DS_CREDIT = 4;           // credits are returned every DS_CREDIT e
 constexpr u32 DS_RF = 8;               // refill takes run at most this many ops ahead (R20)
 constexpr u32 DS_HMIN = 1024;          // heapSize floor of the engine (depth >= 10 > DS_RF)
 constexpr u32 DS_NONE = 0xFFFFFFFFu;
+constexpr u32 DSM_HMIN = 64;           // mixed calls: heapSize floor (nodes 1..63 AVAIL: the levels
+                                       // and the stager's children are never EMPTY)
 
 enum : u32 { MK_A = 1, MK_ASTOP = 2, MK_B = 3, MK_BSTOP = 4 };
 
@@ -75,6 +77,7 @@ struct DsCtl {
   u32 rf_seq;            // takes published
   u32 rf_min[DS_RF], rf_max[DS_RF];
   u32 rf_used;           // ops whose take thread 0 consumed
+  u32 pfs[4];            // mixed calls: R0's prefetch ring of sorted INSERT batches (slots)
   // stager: helper A (LOCK + stage children) and helper B (tasks, write-backs, UNLOCKs) rings
   u32 sq_done;           // staging records published (helper A -> thread 0), one per op
   u32 sq_ret;            // ops whose staging slots thread 0 returned
@@ -264,8 +267,8 @@ struct DsRole {
   __device__ __forceinline__ void load_node(u32 s, u32 n) {
     fence_proxy_async();
     mbar_arrive_expect_tx(&c->lbar, SLOTB);
-    bulk_g2s(BK(s), H.gk + (size_t)n * K, NB, &c->lbar);
-    if (V) bulk_g2s(BV(s), H.gv + (size_t)n * K, NB, &c->lbar);
+    bulk_g2s(BK(s), src_keys<K>(H, n), NB, &c->lbar);
+    if (V) bulk_g2s(BV(s), src_vals<K>(H, n), NB, &c->lbar);
     mbar_wait(&c->lbar, lph);
     lph ^= 1u;
   }
@@ -293,6 +296,11 @@ __device__ __forceinline__ void ds_split(DsRole<K, V>& R, u32 z, u32 w, u32 x, u
 // root and extracts all K keys of it after the heapify, Alg.2 l.4-14 + l.5-6 of Alg.3.)
 __device__ __forceinline__ u64 ds_ops(const HeapArgs& H, const CallArgs& C, int K) {
   const u32 hs = ld_relaxed(H.hdr + H_HS), rs = ld_relaxed(H.hdr + H_RS), ps = ld_relaxed(H.hdr + H_PS);
+  if (C.mode == MODE_MIXED) {  // op pairs (INSERT(K), DELETEMIN(K)) from the call's start
+    if ((rs != (u32)K && rs != 0) || ps != 0 || hs < DSM_HMIN || hs + 1u > H.cap) return 0;
+    const u64 np = C.n_ops / 2, pe = ld_relaxed(C.pair_end);
+    return np < pe ? np : pe;
+  }
   if ((rs != (u32)K && rs != 0) || ps != 0 || hs < DS_HMIN + 2) return 0;
   const u64 full = C.n / (u64)K;
   const u64 room = hs - DS_HMIN;
@@ -451,6 +459,243 @@ __device__ void ds_r0(DsRole<K, V>& R, const u64 m) {
     asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(H.hdr + H_LIN), "l"(lin + m) : "memory");
     c->st[S_KEYS_OUT] += m * (u64)K;
     if (R.C.d_count && m) atomicAdd(R.C.d_count, (ull)(m * (u64)K));
+    *reinterpret_cast<volatile u64*>(R.D.op_base) = m;
+  }
+}
+
+// -----------------------------------------------------------------------------------------
+// R0 of a mixed call: op pairs (INSERT(K), DELETEMIN(K)) in call order (the utilisation
+// workload).  Pair i's INSERT takes the target tar = heapSize + 1 (Alg.1 l.4-6), runs
+// its root section (l.20; the pBuffer is empty and the batch full, so l.26-28 leave both as
+// they are) and its first INSERT_HEAPIFY step at NEXT(root, tar) (l.33), a node R0 holds on
+// chip.  The DELETEMIN that follows takes tar as its refill node (Alg.2 l.5): tar is TARGET,
+// so the DELETEMIN marks it MARKED (l.7-9), the INSERT breaks out at its next check (Alg.1
+// l.31) and puts its items into the root (l.11-13): the refill keys are the INSERT's
+// items after its depth-1 step, heapSize is back at its old value and tar EMPTY again.  That
+// is the interleaving in which the DELETEMIN's root section starts as soon as the INSERT
+// released the root — R0 executes it without touching tar (reading R26).  The
+// DELETEMIN then continues exactly as in ds_r0 (depth-0 step; levels below unchanged).
+// The items arrive sorted (Alg.1 l.2) from bgpq_msort_kernel in H.xk + i*K; they sink by
+// reference (XREF | i) while unchanged, otherwise R0 stores them back there first.
+// -----------------------------------------------------------------------------------------
+template <int K, bool V>
+__device__ void ds_r0_mixed(DsRole<K, V>& R, const u64 m) {
+  DsCtl* c = R.c;
+  const HeapArgs& H = R.H;
+  const CallArgs& C = R.C;
+  const int tid = threadIdx.x;
+  constexpr u32 PF = 3;  // sorted INSERT batches loaded ahead (ring of 4: c->pfs / c->sbar)
+  constexpr u32 NB = DsRole<K, V>::NB;
+  const u32 hs = ld_relaxed(H.hdr + H_HS);
+  const bool rz = ld_relaxed(H.hdr + H_RS) == 0;  // R4: a drained root stays empty
+  const u32 d1 = next_on_path(1u, hs + 1u);         // NEXT(root, tar) of every pair (2 or 3)
+  u32* ns = c->ns;
+  u32* mn = c->mn;
+  u32* mx = c->mx;
+  u32* pend = c->pend;
+  ull lin0 = 0;
+  u32 pfph = 0;                      // sbar parities (thread 0)
+  u32 it = 0, imin = 0, imax = 0;    // thread 0: the INSERT's items (slot, min, max)
+  u32 dirty = 0;                     // thread 0: items differ from H.xk + i*K
+  if (tid == 0) {
+    ns[1] = DS_NONE;
+    for (u32 q = rz ? 2 : 1; q <= 3; ++q) {
+      ns[q] = R.alloc();
+      pend[q] = 0;
+      mn[q] = ld_relaxed(&H.meta[q].kmin);
+      mx[q] = ld_relaxed(&H.meta[q].kmax);
+    }
+    pend[1] = 0;
+    fence_proxy_async();
+    mbar_arrive_expect_tx(&c->lbar, (rz ? 2u : 3u) * DsRole<K, V>::SLOTB);
+    for (u32 q = rz ? 2 : 1; q <= 3; ++q) {
+      bulk_g2s(R.BK(ns[q]), H.gk + (size_t)q * K, NB, &c->lbar);
+      if (V) bulk_g2s(R.BV(ns[q]), H.gv + (size_t)q * K, NB, &c->lbar);
+    }
+    mbar_wait(&c->lbar, R.lph);
+    R.lph ^= 1u;
+    asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(lin0) : "l"(H.hdr + H_LIN) : "memory");
+  }
+  cta_bar<DS_NT>();
+  u32 out_old = DS_NONE;
+  auto output = [&](u64 j, u32 s) {  // op j's K output keys from slot s (TMA bulk store)
+    asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+    R.release(out_old);
+    const u64 pos = j * (u64)K;
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    bulk_s2g(C.out_k + pos, R.BK(s), NB);
+    if (V && C.out_v) bulk_s2g(C.out_v + pos, R.BV(s), NB);
+    asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+    out_old = s;
+  };
+  auto prefetch = [&](u64 k) {  // pair k's sorted items into a fresh slot
+    const u32 s = R.alloc();
+    c->pfs[k % 4] = s;
+    fence_proxy_async();
+    mbar_arrive_expect_tx(&c->sbar[k % 4], DsRole<K, V>::SLOTB);
+    bulk_g2s(R.BK(s), H.xk + (size_t)k * K, NB, &c->sbar[k % 4]);
+    if (V) bulk_g2s(R.BV(s), H.xv + (size_t)k * K, NB, &c->sbar[k % 4]);
+  };
+  if (tid == 0)
+    for (u64 k = 0; k < PF && k < m; ++k) prefetch(k);
+  const ull t_start = R.tnow();
+  for (u64 i = 0; i < m; ++i) {
+    const u64 jd = 2 * i + 1;  // the DELETEMIN's op index (the INSERT is 2i)
+    // ---- INSERT, Alg.1 l.20: (root, items) <- SORT_SPLIT(root, |root|, items, K, |root|)
+    if (tid == 0) {
+      if (i + PF < m) prefetch(i + PF);
+      const ull t1 = R.tnow();
+      mbar_wait(&c->sbar[i % 4], (pfph >> (i % 4)) & 1u);
+      pfph ^= 1u << (i % 4);
+      R.tacc(1, t1);
+      it = c->pfs[i % 4];
+      imin = R.BK(it)[0];
+      imax = R.BK(it)[K - 1];
+      const ull t2 = R.tnow();
+      for (u32 q = 2; q <= 3; ++q)  // op i-1's y1 push must have landed (depth 1 is read below)
+        if (pend[q]) {
+          R.wait_pushed(ns[q]);
+          pend[q] = 0;
+          mn[q] = R.BK(ns[q])[0];
+          mx[q] = R.BK(ns[q])[K - 1];
+        }
+      R.tacc(2, t2);
+      c->st[S_INS_OPS]++;
+      c->st[S_INS_HEAPIFY]++;
+      const u32 ra = rz ? 0u : (mx[1] <= imin) ? 0u : (imax <= mn[1]) ? 1u : 2u;
+      if (ra == 1) {  // the batch lies entirely below the root: swap the contents
+        const u32 t = ns[1]; ns[1] = it; it = t;
+        const u32 a = mn[1], b = mx[1]; mn[1] = imin; mx[1] = imax; imin = a; imax = b;
+      }
+      dirty = ra != 0;
+      c->b[0] = ra;
+      if (ra == 2) { c->b[1] = ns[1]; c->b[2] = it; c->b[3] = R.alloc(); c->b[4] = R.alloc(); }
+    }
+    cta_bar<DS_NT>();
+    if (c->b[0] == 2) {
+      ds_split<K, V>(R, c->b[1], c->b[2], c->b[3], c->b[4]);
+      if (tid == 0) {
+        R.release(ns[1]); R.release(it);
+        ns[1] = c->b[3]; it = c->b[4];
+        mn[1] = R.BK(ns[1])[0]; mx[1] = R.BK(ns[1])[K - 1];
+        imin = R.BK(it)[0]; imax = R.BK(it)[K - 1];
+      }
+    }
+    // ---- INSERT, l.33 at cur = NEXT(root, tar): (Heap[cur], items) <- SORT_SPLIT(Heap[cur], items)
+    if (tid == 0) {
+      const u32 da = (mx[d1] <= imin) ? 0u : (imax <= mn[d1]) ? 1u : 2u;
+      c->st[S_INS_LEVELS]++;
+      c->st[da == 0 ? S_INS_NOOP : da == 1 ? S_INS_SWAP : S_INS_MERGE]++;
+      if (da == 1) {
+        const u32 t = ns[d1]; ns[d1] = it; it = t;
+        const u32 a = mn[d1], b = mx[d1]; mn[d1] = imin; mx[d1] = imax; imin = a; imax = b;
+      }
+      dirty |= da != 0;
+      c->b[0] = da;
+      if (da == 2) { c->b[1] = ns[d1]; c->b[2] = it; c->b[3] = R.alloc(); c->b[4] = R.alloc(); }
+    }
+    cta_bar<DS_NT>();
+    if (c->b[0] == 2) {
+      ds_split<K, V>(R, c->b[1], c->b[2], c->b[3], c->b[4]);
+      if (tid == 0) {
+        R.release(ns[d1]); R.release(it);
+        ns[d1] = c->b[3]; it = c->b[4];
+        mn[d1] = R.BK(ns[d1])[0]; mx[d1] = R.BK(ns[d1])[K - 1];
+        imin = R.BK(it)[0]; imax = R.BK(it)[K - 1];
+      }
+    }
+    // ---- DELETEMIN: the root's keys are its output (Alg.2 l.22), the refill keys are the
+    // INSERT's items (the MARKED hand-off, l.7-12), then Alg.3 at the root as in ds_r0
+    if (tid == 0) {
+      c->st[S_DEL_OPS]++;
+      c->st[S_DEL_REFILL]++;
+      c->st[S_MARKED]++;
+      if (C.lin_ticket) {
+        st_relaxed_u64(reinterpret_cast<u64*>(C.lin_ticket) + 2 * i, lin0 + 2 * i);
+        st_relaxed_u64(reinterpret_cast<u64*>(C.lin_ticket) + jd, lin0 + jd);
+      }
+      st_relaxed(C.op_count + jd, (u32)K);
+      if (!rz) output(jd, ns[1]);
+      const u32 minc = mn[2] < mn[3] ? mn[2] : mn[3];
+      if (imax <= minc) {  // l.4: stop at the root — root <- the refill keys
+        if (rz) output(jd, it);
+        else { ns[1] = it; mn[1] = imin; mx[1] = imax; }
+        R.send((u32)i, MK_ASTOP);
+        c->b[0] = 1;
+      } else {
+        const u32 x = mx[2] > mx[3] ? 2u : 3u, y = 5u - x;  // l.9 (R6: tie -> x = r)
+        const u32 sy = R.alloc();
+        R.arm_slot(sy);
+        R.send((u32)i, MK_A, y, sy);
+        const u32 A = R.alloc(), B = R.alloc();
+        c->b[0] = 0; c->b[1] = ns[2]; c->b[2] = ns[3]; c->b[3] = A; c->b[4] = B;
+        c->b[5] = x; c->b[6] = y; c->b[7] = sy;
+        c->st[S_DEL_LEVELS]++;
+        c->st[(mx[2] <= mn[3] || mx[3] <= mn[2]) ? S_DEL_LR_NOMOVE : S_DEL_LR_MERGE]++;
+      }
+    }
+    cta_bar<DS_NT>();
+    if (c->b[0]) continue;
+    const u32 s2 = c->b[1], s3 = c->b[2], A = c->b[3], B = c->b[4];
+    const ull t3 = R.tnow();
+    ds_split<K, V>(R, s2, s3, A, B);  // l.10
+    if (tid == 0) R.tacc(3, t3);
+    if (tid == 0) {
+      const u32 x = c->b[5], y = c->b[6], sy = c->b[7];
+      R.release(s2); R.release(s3);
+      const u32 ymax = R.BK(A)[K - 1];
+      if (ymax <= imin) {  // l.12 is a swap: root <- Y, the refill keys sink on (by reference)
+        c->st[S_DEL_CY_SWAP]++;
+        if (dirty) {  // the items changed on chip: H.xk + i*K must hold them before the reference
+          asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+          bulk_s2g(H.xk + (size_t)i * K, R.BK(it), NB);
+          if (V) bulk_s2g(H.xv + (size_t)i * K, R.BV(it), NB);
+          asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+          asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+          __threadfence();
+        }
+        R.send((u32)i, MK_B, 0, 0, XREF | (u32)i, imin, imax);
+        R.release(it);
+        if (rz) output(jd, A);
+        else { ns[1] = A; mn[1] = R.BK(A)[0]; mx[1] = ymax; }
+        c->b[15] = 0;
+      } else {  // l.12 merges: (root, C1) <- SORT_SPLIT(refill, Y); C1 into y1's dead HBM copy
+        c->b[11] = it; c->b[12] = R.alloc(); c->b[13] = R.alloc();
+        c->b[15] = 1;
+      }
+      ns[x] = B; mn[x] = R.BK(B)[0]; mx[x] = R.BK(B)[K - 1];
+      ns[y] = sy; pend[y] = 1;
+    }
+    cta_bar<DS_NT>();
+    if (c->b[15]) {
+      const u32 r = c->b[11], lo = c->b[12], hi = c->b[13];
+      ds_split<K, V>(R, r, A, lo, hi);
+      if (tid == 0) {
+        const u32 y = c->b[6];
+        R.store_node(y, hi);
+        __threadfence();
+        R.send((u32)i, MK_B, 0, 0, y, R.BK(hi)[0], R.BK(hi)[K - 1]);
+        if (rz) output(jd, lo);
+        else { ns[1] = lo; mn[1] = R.BK(lo)[0]; mx[1] = R.BK(lo)[K - 1]; }
+        R.release(r); R.release(hi); R.release(A);
+      }
+      cta_bar<DS_NT>();
+    }
+  }
+  // ---- end: the on-chip nodes back to HBM; heapSize is unchanged by every pair
+  if (tid == 0) {
+    R.tacc(0, t_start);
+    for (u32 q = 2; q <= 3; ++q)
+      if (pend[q]) { R.wait_pushed(ns[q]); pend[q] = 0; mn[q] = R.BK(ns[q])[0]; mx[q] = R.BK(ns[q])[K - 1]; }
+    asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+    for (u32 q = rz ? 2 : 1; q <= 3; ++q) {
+      R.store_node(q, ns[q]);
+      st_relaxed(&H.meta[q].kmin, mn[q]);
+      st_relaxed(&H.meta[q].kmax, mx[q]);
+    }
+    asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(H.hdr + H_LIN), "l"(lin0 + 2 * m) : "memory");
+    st_relaxed(H.hdr + H_FETCH, (u32)(2 * m));  // the lock engine continues at op 2m
+    c->st[S_KEYS_OUT] += m * (u64)K;
     *reinterpret_cast<volatile u64*>(R.D.op_base) = m;
   }
 }
@@ -884,14 +1129,17 @@ __global__ void __cluster_dims__(DS_CL, 1, 1) __launch_bounds__(DS_BLOCK, 1)
     const bool stager = R.rank == DS_CL - 1;
     if (threadIdx.x >= DS_NT) {
       if (threadIdx.x == DS_NT) {
-        if (R.rank == 0) ds_r0_helper<K, V>(R, m);
+        if (R.rank == 0) { if (C.mode != MODE_MIXED) ds_r0_helper<K, V>(R, m); }
         else if (stager) ds_stage_helper<K, V>(R, m);
       } else if (threadIdx.x == DS_NT + 32 && stager) {
         ds_wb_helper<K, V>(R);
       }
     } else {
       if (m) {
-        if (R.rank == 0) ds_r0<K, V>(R, m);
+        if (R.rank == 0) {
+          if (C.mode == MODE_MIXED) ds_r0_mixed<K, V>(R, m);
+          else ds_r0<K, V>(R, m);
+        }
         else if (stager) ds_stager<K, V>(R, m);
         else ds_level<K, V>(R, m);
       } else if (threadIdx.x == 0 && R.rank == 0) {
@@ -915,5 +1163,55 @@ __global__ void __cluster_dims__(DS_CL, 1, 1) __launch_bounds__(DS_BLOCK, 1)
   }
   dt_walkers<K, V, DS_NT>(H, C, D, smem_raw);
 }
+
+// Mixed calls on the cluster engine, step 1: Alg.1 l.2 (Sort(items), done before the root is
+// locked) for every op pair (INSERT(K), DELETEMIN(K)) at the call's start, into H.xk + p*K, and
+// the first op pair of another shape (atomicMin into *C.pair_end, preset to all-ones).  Pairs
+// after that one are left unsorted (the per-node-lock engine executes them).
+template <int K, bool V, int NT>
+__global__ void __launch_bounds__(NT, 1) bgpq_msort_kernel(HeapArgs H, CallArgs C) {
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  u32* ak = reinterpret_cast<u32*>(smem_raw);
+  u32* tk = ak + K;
+  u32* av = V ? tk + K : nullptr;
+  u32* tv = V ? av + K : nullptr;
+  u32* pe = const_cast<u32*>(C.pair_end);
+  const u64 np = C.n_ops / 2;
+  __shared__ u32 go;
+  for (u64 p = blockIdx.x; p < np; p += gridDim.x) {
+    const u64 j = 2 * p;
+    if (threadIdx.x == 0) {  // one thread decides: the CTA leaves the loop as a whole
+      go = 0;
+      if (p < *reinterpret_cast<volatile const u32*>(pe)) {
+        if (C.op_types[j] == 0 && C.op_types[j + 1] == 1 && C.op_sizes[j] == (u32)K && C.op_sizes[j + 1] == (u32)K)
+          go = 1;
+        else
+          atomicMin(pe, (u32)p);
+      }
+    }
+    cta_bar<NT>();
+    if (!go) break;
+    const u32* ik = C.in_k + C.in_off[j];
+    const u32* iv = C.in_v ? C.in_v + C.in_off[j] : nullptr;
+    for (int e = threadIdx.x; e < K; e += NT) {
+      ak[e] = ik[e];
+      if (V) av[e] = iv ? iv[e] : 0u;
+    }
+    cta_bar<NT>();
+    const bool swapped = cta_sort<K, NT, V>(ak, av, K, tk, tv);
+    cta_bar<NT>();
+    const uint4* sk = reinterpret_cast<const uint4*>(swapped ? tk : ak);
+    uint4* dk = reinterpret_cast<uint4*>(H.xk + p * (u64)K);
+    for (int e = threadIdx.x; e < K / 4; e += NT) dk[e] = sk[e];
+    if (V) {
+      const uint4* sv = reinterpret_cast<const uint4*>(swapped ? tv : av);
+      uint4* dv = reinterpret_cast<uint4*>(H.xv + p * (u64)K);
+      for (int e = threadIdx.x; e < K / 4; e += NT) dv[e] = sv[e];
+    }
+    cta_bar<NT>();
+  }
+}
+template <int K, bool V>
+constexpr size_t msort_smem_bytes() { return (size_t)2 * K * 4 * (V ? 2 : 1); }
 
 }  // namespace bgpqd

@@ -76,6 +76,14 @@ cudaError_t ds_launch(int grid, const HeapArgs& H, const CallArgs& C, const DtAr
   }
   return cudaErrorInvalidValue;
 }
+cudaError_t ms_launch(int grid, const HeapArgs& H, const CallArgs& C, cudaStream_t s) {
+  if constexpr (kDs) {
+    static_assert(!kDs || msort_smem_bytes<K, V>() <= 48 * 1024, "msort fits the default smem");
+    bgpq_msort_kernel<K, V, NT><<<grid, NT, msort_smem_bytes<K, V>(), s>>>(H, C);
+    return cudaGetLastError();
+  }
+  return cudaErrorInvalidValue;
+}
 cudaError_t pipe_prepare(int* occ) {
   if constexpr (kPipe) {
     auto kern = bgpq_ins_pipe2_kernel<K, V, NT>;
@@ -97,6 +105,7 @@ cudaError_t pipe_launch(int grid, const HeapArgs& H, const PipeArgs& P, const Ca
 const KTable kTable = {kLocks ? locks_prepare : nullptr, kLocks ? locks_launch : nullptr,
                        kDt ? dt_prepare : nullptr,       kDt ? dt_launch : nullptr,
                        kDs ? ds_prepare : nullptr,       kDs ? ds_launch : nullptr,
+                       kDs ? ms_launch : nullptr,
                        kPipe ? pipe_prepare : nullptr,   kPipe ? pipe_launch : nullptr};
 
 }  // namespace

@@ -26,6 +26,10 @@ struct KTable {
   // the number of co-resident clusters in *clusters (0 if the engine cannot run)
   cudaError_t (*ds_prepare)(int sm_count, int* clusters);
   cudaError_t (*ds_launch)(int grid, const HeapArgs& H, const CallArgs& C, const DtArgs& D, cudaStream_t s);
+  // mixed calls on the cluster engine: Sort(items) of the call's leading (INSERT(K),
+  // DELETEMIN(K)) pairs into H.xk and the pair count into *C.pair_end (bgpq_dsys.cuh); the
+  // pairs then run on ds_launch with C.mode = MODE_MIXED
+  cudaError_t (*ms_launch)(int grid, const HeapArgs& H, const CallArgs& C, cudaStream_t s);
   // insert calls: level pipeline (bgpq_pipe2.cuh)
   cudaError_t (*pipe_prepare)(int* occ);
   cudaError_t (*pipe_launch)(int grid, const HeapArgs& H, const PipeArgs& P, const CallArgs& C, cudaStream_t s);

@@ -139,8 +139,8 @@ struct OpL {
     if (threadIdx.x == 0) {
       fence_proxy_async();
       mbar_arrive_expect_tx(&ctl->bar, V ? 2u * NBYTES : NBYTES);
-      bulk_g2s(BK(s), H.gk + (size_t)node * K, NBYTES, &ctl->bar);
-      if (V) bulk_g2s(BV(s), H.gv + (size_t)node * K, NBYTES, &ctl->bar);
+      bulk_g2s(BK(s), src_keys<K>(H, node), NBYTES, &ctl->bar);
+      if (V) bulk_g2s(BV(s), src_vals<K>(H, node), NBYTES, &ctl->bar);
     }
     mbar_wait(&ctl->bar, mphase);
     mphase ^= 1u;
