@@ -140,8 +140,7 @@ int ensure_pipe(bgpq* q) {
   ok = ok && cudaMalloc(&P.sbk, PIPE_NSB * kb) == cudaSuccess;
   ok = ok && cudaMalloc(&P.sready, PIPE_NSB * sizeof(u32)) == cudaSuccess;
   ok = ok && cudaMalloc(&P.rk, (size_t)PIPE_MAXL * PIPE_NL * kb) == cudaSuccess;
-  ok = ok && cudaMalloc(&P.rhdr, (size_t)PIPE_MAXL * PIPE_NL * 4 * sizeof(u32)) == cudaSuccess;
-  ok = ok && cudaMalloc(&P.rflag, (size_t)PIPE_MAXL * PIPE_NL * sizeof(u32)) == cudaSuccess;
+  ok = ok && cudaMalloc(&P.rflag, (size_t)PIPE_MAXL * PIPE_NL * sizeof(u64)) == cudaSuccess;
   if (V) {
     ok = ok && cudaMalloc(&P.sbv, PIPE_NSB * kb) == cudaSuccess;
     ok = ok && cudaMalloc(&P.rv, (size_t)PIPE_MAXL * PIPE_NL * kb) == cudaSuccess;
@@ -290,7 +289,7 @@ int run_call(bgpq* q, const CallArgs& C, cudaStream_t s) {
     const PipeArgs& P = q->pipe;
     bool ok = cudaMemsetAsync(P.ctl, 0, PC_WORDS * sizeof(u32), s) == cudaSuccess;
     ok = ok && cudaMemsetAsync(P.sready, 0, PIPE_NSB * sizeof(u32), s) == cudaSuccess;
-    ok = ok && cudaMemsetAsync(P.rflag, 0, (size_t)PIPE_MAXL * PIPE_NL * sizeof(u32), s) == cudaSuccess;
+    ok = ok && cudaMemsetAsync(P.rflag, 0, (size_t)PIPE_MAXL * PIPE_NL * sizeof(u64), s) == cudaSuccess;
     if (!ok) return fail(BGPQ_ECUDA);
     if (counted(ktab(q)->pipe_launch(q->pipe_grid, heap_args(q), P, C, s)) != cudaSuccess) return fail(BGPQ_ECUDA);
     return BGPQ_OK;
@@ -397,8 +396,9 @@ void bgpq_destroy(bgpq_t* q) {
   cudaFree(q->pair_end);
   cudaFree(q->dt.ctl);
   PipeArgs& P = q->pipe;
-  u32* pbufs[] = {P.ctl, P.sbk, P.sbv, P.sready, P.rk, P.rv, P.rhdr, P.rflag};
+  u32* pbufs[] = {P.ctl, P.sbk, P.sbv, P.sready, P.rk, P.rv};
   for (u32* b : pbufs) cudaFree(b);
+  cudaFree(P.rflag);
   delete q;
 }
 

@@ -58,6 +58,15 @@ constexpr size_t pipe2_smem_bytes() {
 }
 
 __device__ __forceinline__ u32 vld(const u32* p) { return *reinterpret_cast<const volatile u32*>(p); }
+// back-off of the pipeline's hot polls (flags, flow control, ring room): a short sleep keeps the
+// single-thread pollers from taking issue slots from the compute warps of their SM (measured:
+// C2 insert 148 ms with 32 ns vs 160 ms with no sleep)
+#ifndef BGPQ_P2_SLEEP
+#define BGPQ_P2_SLEEP 32
+#endif
+__device__ __forceinline__ void p2_pause() {
+  if (BGPQ_P2_SLEEP) __nanosleep(BGPQ_P2_SLEEP);
+}
 
 template <int K, bool V, int NT>
 struct Pipe2 {
@@ -103,7 +112,7 @@ struct Pipe2 {
     const u32 h = pc->rq_head;
     if (h - vld(&pc->rq_done) >= P2_RQ) {
       const ull t0 = (C.debug & 16384u) ? clock64() : 0ull;
-      while (h - vld(&pc->rq_done) >= P2_RQ) __nanosleep(32);
+      while (h - vld(&pc->rq_done) >= P2_RQ) p2_pause();
       if (C.debug & 16384u) th2 += clock64() - t0;
     }
     u32* e = pc->rq[h % P2_RQ];
@@ -130,33 +139,29 @@ struct Pipe2 {
     if (threadIdx.x == 0 && (C.debug & 128u) && !(C.debug & 65536u)) twait += clock64() - t0;
     tar = pc->ent[e][0]; end = pc->ent[e][1]; is = pc->ent[e][2]; ns = pc->ent[e][3];
     cta_bar<NT>();
-    if (threadIdx.x == 0) st_rel_cta(&pc->icons, m + 1u);
+    if (threadIdx.x == 0) {
+      st_rel_cta(&pc->icons, m + 1u);
+      // the entry's ring slot may be reused by the sender at once (relaxed: its TMA load into
+      // shared memory completed before the wait above returned)
+      st_relaxed(mycons, m + 1u);
+    }
   }
+  u32* mycons;  // this stage's consumption counter read by its sender (P.ctl word)
 
   // ======================================================================================
   // H1 of a level stage l (l >= 1): prefetch messages m = 0, 1, ... from ring l
   // ======================================================================================
   __device__ void h1_level(u32 l) {
-    u32 last_a = 0, nplace = 0, last_cons = 0;
+    u32 last_a = 0, nplace = 0;
     for (u32 m = 0;; ++m) {
       const u32 e = m % P2_PIN;
-      while (m - vld(&pc->icons) >= P2_PIN) __nanosleep(32);
+      while (m - vld(&pc->icons) >= P2_PIN) p2_pause();
       (void)ld_acq_cta(&pc->icons);
       const u32 slot = m % PIPE_NL;
-      const u32* f = P.rflag + (size_t)l * PIPE_NL + slot;
-      while (ld_acquire(f) != m + 1) __nanosleep(32);
-      const u32* hd = P.rhdr + ((size_t)l * PIPE_NL + slot) * 4;
-      const u32 tar = ld_relaxed(hd + 0), end = ld_relaxed(hd + 1);
-      if (C.debug & 8192u) {  // test switch: the previous message's load landed, release it
-        if (m > 0) {
-          mbar_wait(&pc->ibar[(m - 1) % P2_PIN], ((m - 1) / P2_PIN) & 1u);
-          st_release(cons(l), m);
-        }
-      } else {  // ring slots of the messages the compute threads consumed (their loads landed)
-                // may be reused — no wait on the previous message's TMA
-        const u32 done = vld(&pc->icons);
-        if (done != last_cons) { st_release(cons(l), done); last_cons = done; }
-      }
+      const u64* f = P.rflag + (size_t)l * PIPE_NL + slot;
+      u64 w;  // one acquire load: the message index and its header {tar, end}
+      while ((u32)(w = ld_acquire_u64(f)) != m + 1) p2_pause();
+      const u32 tar = (u32)(w >> 32) & 0x7FFFFFFFu, end = (u32)(w >> 63);
       pc->ent[e][0] = tar; pc->ent[e][1] = end; pc->ent[e][2] = P2_NONE; pc->ent[e][3] = P2_NONE;
       if (end) {
         st_release(cons(l), m + 1);
@@ -202,22 +207,17 @@ struct Pipe2 {
 
   // H1 of the root stage: prefetch sorted batches j = 0, 1, ...
   __device__ void h1_root() {
-    u32 last_cons = 0;
     const bool tm = (C.debug & 128u) != 0;
     ull w_icons = 0, w_ready = 0, w_alloc = 0;
     for (u32 j = 0; j < (u32)C.n_ops; ++j) {
       const u32 e = j % P2_PIN;
       ull t0 = tm ? clock64() : 0;
-      while (j - vld(&pc->icons) >= P2_PIN) __nanosleep(32);
+      while (j - vld(&pc->icons) >= P2_PIN) p2_pause();
       (void)ld_acq_cta(&pc->icons);
       if (tm) { const ull t = clock64(); w_icons += t - t0; t0 = t; }
       const u32 slot = j % PIPE_NSB;
-      while (ld_acquire(P.sready + slot) != j + 1) __nanosleep(32);
+      while (ld_acquire(P.sready + slot) != j + 1) p2_pause();
       if (tm) { const ull t = clock64(); w_ready += t - t0; t0 = t; }
-      {  // the sorters may reuse the slots of the batches the root consumed (loads landed)
-        const u32 done = vld(&pc->icons);
-        if (done != last_cons) { st_release(P.ctl + PC_ROOTCONS, done); last_cons = done; }
-      }
       const u32 is = alloc();
       if (tm) { const ull t = clock64(); w_alloc += t - t0; t0 = t; }
       pc->ent[e][0] = op_size(j); pc->ent[e][1] = 0; pc->ent[e][2] = is; pc->ent[e][3] = P2_NONE;
@@ -243,16 +243,22 @@ struct Pipe2 {
     constexpr u32 D = P2_H2D;
     u32 seen = 0, nplaced = 0, inflight = 0, head_i = 0;
     u32 cache_l = P2_NONE, cache_c = 0;
-    auto retire = [&](u32 keep) {  // complete the oldest requests until <= keep are in flight
-      while (inflight > keep) {
-        if (keep == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
-        else if (inflight - 1 == 1) asm volatile("cp.async.bulk.wait_group 1;" ::: "memory");
-        else if (inflight - 1 == 2) asm volatile("cp.async.bulk.wait_group 2;" ::: "memory");
-        else asm volatile("cp.async.bulk.wait_group 3;" ::: "memory");
+    const bool tm = (C.debug & 262144u) != 0;  // debug: H2 flow-control / wait_group / publish cycles
+    ull w_fc = 0, w_wg = 0, w_pub = 0;
+    auto retire = [&](u32 keep) {  // more than `keep` requests in flight: complete all of them
+      if (inflight <= keep) return;
+      const ull t0 = tm ? clock64() : 0ull;
+      asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+      const ull t1 = tm ? clock64() : 0ull;
+      if (tm) w_wg += t1 - t0;
+      // one proxy fence and one release fence publish the whole batch: every request's bulk
+      // data is complete and ordered before the relaxed flag / metadata stores below
+      asm volatile("fence.proxy.async.global;" ::: "memory");
+      asm volatile("fence.acq_rel.gpu;" ::: "memory");
+      while (inflight) {
         const u32* f = pc->fq[head_i % D];
         const u32 type = f[0], a = f[1], b = f[2], c = f[3];
         if (f[4] != P2_NONE) release(f[4]);  // the smem source was read
-        asm volatile("fence.proxy.async.global;" ::: "memory");
         if (type == P2_WB) {
           st_relaxed(&H.meta[a].kmin, f[5]);
           st_relaxed(&H.meta[a].kmax, f[6]);
@@ -260,24 +266,31 @@ struct Pipe2 {
             st_relaxed(&H.meta[a].state, ST_AVAIL);
             st_rel_cta(&pc->place_done, ++nplaced);
           }
-        } else {  // SEND / END: header, then the flag (release)
+        } else {  // SEND / END: the flag word with the header
           const u32 l = a >> 8, m = b, rs = m % PIPE_NL;
-          u32* hd = P.rhdr + ((size_t)l * PIPE_NL + rs) * 4;
-          if (type == P2_SEND) { st_relaxed(hd + 0, c); st_relaxed(hd + 1, 0u); }
-          else { st_relaxed(hd + 0, 0u); st_relaxed(hd + 1, 1u); }
-          st_release(P.rflag + (size_t)l * PIPE_NL + rs, m + 1);
+          const u64 hdr = type == P2_SEND ? (u64)(c & 0x7FFFFFFFu) : (u64)1u << 31;
+          st_relaxed_u64(P.rflag + (size_t)l * PIPE_NL + rs, (hdr << 32) | (u64)(m + 1));
         }
         ++head_i;
         --inflight;
         ++seen;
-        st_rel_cta(&pc->rq_done, seen);
+      }
+      st_rel_cta(&pc->rq_done, seen);
+      if (tm) w_pub += clock64() - t1;
+    };
+    auto report = [&]() {
+      const u32 b = blockIdx.x - ((C.debug & 524288u) ? 8u : 0u);  // debug 524288: stages 8..23
+      if (tm && b < 16) {
+        ull* tms = reinterpret_cast<ull*>(H.hdr + H_TIME);
+        atomicAdd(tms + b, w_fc + (w_wg << 32));   // low: flow control, high: wait_group (cycles >> 0)
+        atomicAdd(tms + 16 + b, w_pub);
       }
     };
     u32 issued = 0;
     for (;;) {
       while (vld(&pc->rq_head) == issued) {
         if (inflight) retire(0);
-        else __nanosleep(32);
+        else p2_pause();
       }
       (void)ld_acq_cta(&pc->rq_head);
       const u32* e = pc->rq[issued % P2_RQ];
@@ -287,6 +300,7 @@ struct Pipe2 {
         ++issued;
         ++seen;
         st_rel_cta(&pc->rq_done, seen);
+        report();
         return;
       }
       retire((C.debug & 4096u) ? 0u : D - 1);  // room for one more group (debug 4096: one at a time)
@@ -300,13 +314,15 @@ struct Pipe2 {
       } else {  // P2_SEND (a = level << 8 | slot, b = message, c = tar) / P2_END
         const u32 l = a >> 8, m = b;
         const u32 rs = m % PIPE_NL;
+        const ull tf = tm ? clock64() : 0ull;
         if (m >= PIPE_NL) {  // flow control: the receiver consumed the slot's previous message
           if (cache_l != l) { cache_l = l; cache_c = 0; }
           while (cache_c < m + 1 - PIPE_NL) {
             cache_c = ld_acquire(cons(l));
-            if (cache_c < m + 1 - PIPE_NL) __nanosleep(64);
+            if (cache_c < m + 1 - PIPE_NL) p2_pause();
           }
         }
+        if (tm) w_fc += clock64() - tf;
         if (type == P2_SEND) {
           const u32 s = a & 0xFFu;
           f[4] = s;
@@ -554,13 +570,15 @@ __global__ void __launch_bounds__(NT + 64, 1) bgpq_ins_pipe2_kernel(HeapArgs H, 
     if (threadIdx.x == NT + 32) p.h2_loop();
     return;
   }
+  p.mycons = b == 0 ? P.ctl + PC_ROOTCONS : p.cons(b);
   const ull t0 = clock64();
   if (b == 0) p.root_stage();
   else p.level_stage(b);
-  if (threadIdx.x == 0 && (C.debug & 128u) && b < 16) {
+  const u32 bt = b - ((C.debug & 524288u) ? 8u : 0u);  // debug 524288: stages 8..23
+  if (threadIdx.x == 0 && (C.debug & 128u) && !(C.debug & 262144u) && bt < 16) {
     ull* tms = reinterpret_cast<ull*>(H.hdr + H_TIME);
-    atomicAdd(tms + b, p.twait);
-    atomicAdd(tms + 16 + b, (C.debug & 16384u) ? p.th2 : clock64() - t0);
+    atomicAdd(tms + bt, p.twait);
+    atomicAdd(tms + 16 + bt, (C.debug & 16384u) ? p.th2 : clock64() - t0);
   }
   if (threadIdx.x == 0) {
     ull* stat = reinterpret_cast<ull*>(H.hdr + H_STAT);
