@@ -49,6 +49,11 @@ constexpr u32 DSM_HMIN = 64;           // mixed calls: heapSize floor (nodes 1..
                                        // and the stager's children are never EMPTY)
 
 enum : u32 { MK_A = 1, MK_ASTOP = 2, MK_B = 3, MK_BSTOP = 4 };
+// MK_A flag: every level above that swaps its (cur, y) split (l.12) passes the refill keys R
+// on unchanged (src, [cmin, cmax] of the message), and the walk does not stop above given
+// that.  A level whose own step then provably swaps commits it without message b (early
+// commit, see ds_level).
+constexpr u32 MA_EARLY = 1;
 
 
 struct __align__(16) DsMsg {
@@ -196,7 +201,7 @@ struct DsRole {
     DsMsg m;
     volatile DsMsg* pm = &c->inbox[e];
     m.op = pm->op; m.kind = pm->kind; m.y = pm->y; m.slot = pm->slot;
-    m.src = pm->src; m.cmin = pm->cmin; m.cmax = pm->cmax;
+    m.src = pm->src; m.cmin = pm->cmin; m.cmax = pm->cmax; m.pad = pm->pad;
     ++in_seq;
     arm_inbox(e);  // for the message DS_RING entries later
     if (in_seq % DS_CREDIT == 0) {  // credit back to the sender (its staging entries are free too)
@@ -209,13 +214,13 @@ struct DsRole {
   }
   // ---- send to the level below (thread 0)
   __device__ __forceinline__ void send(u32 op, u32 kind, u32 y = 0, u32 slot = 0, u32 src = 0, u32 cmin = 0,
-                                       u32 cmax = 0) {
+                                       u32 cmax = 0, u32 flags = 0) {
     const ull t0 = tnow();
     while (out_seq - *reinterpret_cast<volatile u32*>(&c->consumed) >= DS_RING - DS_CREDIT) {}
     const u32 e = out_seq % DS_RING;
     const u32 dst = rank + 1;
     DsMsg& m = c->stage[e];
-    m.op = op; m.kind = kind; m.y = y; m.slot = slot; m.src = src; m.cmin = cmin; m.cmax = cmax; m.pad = 0;
+    m.op = op; m.kind = kind; m.y = y; m.slot = slot; m.src = src; m.cmin = cmin; m.cmax = cmax; m.pad = flags;
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
     bulk_s2cl(cl_map(&c->inbox[e], dst), &m, (u32)sizeof(DsMsg), cl_map(&c->inbar[e], dst));
     asm volatile("cp.async.bulk.commit_group;" ::: "memory");
@@ -236,9 +241,10 @@ struct DsRole {
     ++out_seq2;
     tacc(5, t0);
   }
-  __device__ __forceinline__ void send_path(u32 op, u32 kind, u32 y = 0, u32 slot = 0) {
+  __device__ __forceinline__ void send_path(u32 op, u32 kind, u32 y = 0, u32 slot = 0, u32 src = 0, u32 cmin = 0,
+                                            u32 cmax = 0, u32 flags = 0) {
     if (rank + 2 == (u32)DS_CL) send_a2(op, kind, y, slot);
-    else send(op, kind, y, slot);
+    else send(op, kind, y, slot, src, cmin, cmax, flags);
   }
   // ---- slots the level below pushes into: armed when designated, disarmed if no push comes
   __device__ __forceinline__ void arm_slot(u32 s) { mbar_arrive_expect_tx(&c->slotbar[s], SLOTB); }
@@ -393,7 +399,7 @@ __device__ void ds_r0(DsRole<K, V>& R, const u64 m) {
         const u32 x = mx[2] > mx[3] ? 2u : 3u, y = 5u - x;  // l.9 (R6: tie -> x = r)
         const u32 sy = R.alloc();  // y1's new content arrives here from R1
         R.arm_slot(sy);
-        R.send((u32)i, MK_A, y, sy);
+        R.send((u32)i, MK_A, y, sy, t, rmin, rmax, MA_EARLY);
         const u32 A = R.alloc(), B = R.alloc();
         c->b[0] = 0; c->b[1] = ns[2]; c->b[2] = ns[3]; c->b[3] = A; c->b[4] = B;
         c->b[5] = x; c->b[6] = y; c->b[7] = sy; c->b[8] = t; c->b[9] = rmin; c->b[10] = rmax;
@@ -626,7 +632,8 @@ __device__ void ds_r0_mixed(DsRole<K, V>& R, const u64 m) {
         const u32 x = mx[2] > mx[3] ? 2u : 3u, y = 5u - x;  // l.9 (R6: tie -> x = r)
         const u32 sy = R.alloc();
         R.arm_slot(sy);
-        R.send((u32)i, MK_A, y, sy);
+        // early commit below (MA_EARLY) only while the items are still the HBM copy H.xk + i*K
+        R.send((u32)i, MK_A, y, sy, XREF | (u32)i, imin, imax, dirty ? 0u : MA_EARLY);
         const u32 A = R.alloc(), B = R.alloc();
         c->b[0] = 0; c->b[1] = ns[2]; c->b[2] = ns[3]; c->b[3] = A; c->b[4] = B;
         c->b[5] = x; c->b[6] = y; c->b[7] = sy;
@@ -759,6 +766,7 @@ __device__ void ds_level(DsRole<K, V>& R, const u64 m) {
   }
   cta_bar<DS_NT>();
   u32 push_old = DS_NONE;  // slot whose push may still be reading it
+  u32 a_src = 0, a_cmin = 0, a_cmax = 0, early = 0;  // thread 0: the path message's refill-key info
   const ull t_start = R.tnow();
   for (u64 i = 0; i < m; ++i) {
     if (tid == 0) {
@@ -783,14 +791,19 @@ __device__ void ds_level(DsRole<K, V>& R, const u64 m) {
         }
         R.tacc(2, t2);
         const u32 x = mx[jl] > mx[jr] ? l : r, y = l + r - x;  // l.9 (R6)
+        const u32 minc = mn[jl] < mn[jr] ? mn[jl] : mn[jr];
+        // early commit (MA_EARLY): the carried keys are R = [a.cmin, a.cmax] at a.src if every
+        // level above swapped; with R the walk does not stop here (l.4) iff a.cmax > minc
+        a_src = a.src; a_cmin = a.cmin; a_cmax = a.cmax;
+        early = !(R.C.debug & 1048576u) && (a.pad & MA_EARLY) && a.cmax > minc;  // debug 1048576: off
         const u32 sy = R.alloc();  // y's new content arrives here from the level below
         R.arm_slot(sy);
-        R.send_path((u32)i, MK_A, y, sy);
+        R.send_path((u32)i, MK_A, y, sy, a.src, a.cmin, a.cmax, early ? MA_EARLY : 0u);
         const u32 A = R.alloc(), B = R.alloc();
         c->b[1] = ns[jl]; c->b[2] = ns[jr]; c->b[3] = A; c->b[4] = B; c->b[5] = x; c->b[6] = y;
         c->b[7] = sy; c->b[9] = a.slot;
         c->b[10] = (mx[jl] <= mn[jr] || mx[jr] <= mn[jl]) ? 1u : 0u;
-        c->b[13] = mn[jl] < mn[jr] ? mn[jl] : mn[jr];
+        c->b[13] = minc;
       }
     }
     cta_bar<DS_NT>();
@@ -802,13 +815,35 @@ __device__ void ds_level(DsRole<K, V>& R, const u64 m) {
       R.tacc(3, t3);
       const u32 x = c->b[5], y = c->b[6], sy = c->b[7], up = c->b[9];
       const u32 minc = c->b[13];
+      c->b[14] = 0;
+      if (early && R.BK(A)[K - 1] <= a_cmin) {
+        // Early commit.  max(Y_d) <= min(R) implies max(Y_k) <= min(R) at every level k above
+        // (max(Y_k) <= max(y_k+1) <= min(children of y_k+1) <= max(Y_k+1), heap order), so every
+        // (cur, y) split above was a swap passing R on unchanged, and so is this one: cur <- Y
+        // is final now (pushed up before the level above's message b arrives), R sinks on.
+        asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+        R.release(push_old);
+        c->st[S_DEL_LEVELS]++;
+        c->st[c->b[10] ? S_DEL_LR_NOMOVE : S_DEL_LR_MERGE]++;
+        c->st[S_DEL_CY_SWAP]++;
+        const u32 jx = x - base, jy = y - base;
+        R.release(sl); R.release(sr);
+        ns[jx] = B; mn[jx] = R.BK(B)[0]; mx[jx] = R.BK(B)[K - 1];
+        ns[jy] = sy; pend[jy] = 1;
+        R.push_up(A, up);
+        push_old = A;
+        R.send((u32)i, MK_B, 0, 0, a_src, a_cmin, a_cmax);
+        const ull t4 = R.tnow();
+        const DsMsg b = R.recv();  // the level above's message b, consumed in order
+        R.tacc(4, t4);
+        if (b.kind != MK_B || b.src != a_src) __trap();  // contradicts the argument above
+      } else {
       const ull t4 = R.tnow();
       const DsMsg b = R.recv();  // the carried keys of cur (l.12) from the level above
       R.tacc(4, t4);
       asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");  // the previous push's read
       R.release(push_old);
       push_old = DS_NONE;
-      c->b[14] = 0;
       if (b.kind == MK_BSTOP) {  // the walk stopped above after all: drop the speculative split
         R.release(A); R.release(B);
         R.disarm_slot(sy);
@@ -841,6 +876,7 @@ __device__ void ds_level(DsRole<K, V>& R, const u64 m) {
           R.load_node(cs, b.src);
           c->b[14] = 1; c->b[4] = cs; c->b[5] = lo; c->b[6] = hi; c->b[7] = y; c->b[9] = up; c->b[12] = A;
         }
+      }
       }
     }
     cta_bar<DS_NT>();
