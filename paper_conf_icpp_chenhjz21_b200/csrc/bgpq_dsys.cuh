@@ -1059,8 +1059,10 @@ __device__ void ds_stage_helper(DsRole<K, V>& R, const u64 m) {
     } else {
       const u32 n0 = 2u * y, n1 = n0 + 1u;
       const u32 s0 = DS_NSLOT - 8 + 2 * (k % 4), s1 = s0 + 1;
+      const ull tl = R.tnow();
       lock_acquire(&H.meta[n0].lock);  // l.3: LOCK(l); LOCK(r)
       lock_acquire(&H.meta[n1].lock);
+      R.tacc(1, tl);  // timers: the stager's "wait-above" column = helper A's LOCK time
       fence_proxy_async();
       u64* bar = &c->sbar[k % 4];  // thread 0 waits for the data; this helper moves on
       mbar_arrive_expect_tx(bar, 2u * DsRole<K, V>::SLOTB);
@@ -1070,8 +1072,11 @@ __device__ void ds_stage_helper(DsRole<K, V>& R, const u64 m) {
         bulk_g2s(R.BV(s0), H.gv + (size_t)n0 * K, DsRole<K, V>::NB, bar);
         bulk_g2s(R.BV(s1), H.gv + (size_t)n1 * K, DsRole<K, V>::NB, bar);
       }
-      c->stg_min[q][0] = ld_relaxed(&H.meta[n0].kmin); c->stg_max[q][0] = ld_relaxed(&H.meta[n0].kmax);
-      c->stg_min[q][1] = ld_relaxed(&H.meta[n1].kmin); c->stg_max[q][1] = ld_relaxed(&H.meta[n1].kmax);
+      u32 st0, st1, mn0, mx0, mn1, mx1;
+      meta_load(&H.meta[n0], st0, mn0, mx0);
+      meta_load(&H.meta[n1], st1, mn1, mx1);
+      c->stg_min[q][0] = mn0; c->stg_max[q][0] = mx0;
+      c->stg_min[q][1] = mn1; c->stg_max[q][1] = mx1;
       c->stg_y[q] = y;
       c->stg_up[q] = up;
     }
@@ -1108,6 +1113,7 @@ __device__ void ds_wb_helper(DsRole<K, V>& R) {
         st_relaxed(&H.meta[e[3]].lock, 0u);
       }
     } else if (kind == WQ_WB) {  // Alg.3 l.10-11: x <- X, UNLOCK(x)
+      const ull tw = R.tnow();
       const u32 x = e[1], B = e[2];
       asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
       bulk_s2g(H.gk + (size_t)x * K, R.BK(B), DsRole<K, V>::NB);
@@ -1120,6 +1126,7 @@ __device__ void ds_wb_helper(DsRole<K, V>& R) {
       asm volatile("fence.acq_rel.gpu;" ::: "memory");
       st_relaxed(&H.meta[x].lock, 0u);
       atomicOr(&c->wb_free, 1u << B);
+      R.tacc(5, tw);  // timers: the stager's "sends" column = helper B's write-back time
     }
     ++seen;
     st_rel_cta(&c->wq_done, seen);

@@ -839,9 +839,7 @@ __device__ __forceinline__ void lock_warp(OpL<K, V, NT>& op) {
         const ull t0 = op.timing ? clock64() : 0;
         lock_acquire(op.lk(n));
         if (op.timing) op.tm[LT_P_LOCKWAIT] += clock64() - t0;
-        stv[q] = ld_relaxed(op.stp(n));
-        mn[q] = ld_relaxed(&op.H.meta[n].kmin);
-        mx[q] = ld_relaxed(&op.H.meta[n].kmax);
+        meta_load(&op.H.meta[n], stv[q], mn[q], mx[q]);
         if (force || stv[q] == ST_AVAIL) bytes += V ? 2u * NB : NB;
       }
       for (int q = 0; q < 2; ++q) { c->p_st[q] = stv[q]; c->p_min[q] = mn[q]; c->p_max[q] = mx[q]; }

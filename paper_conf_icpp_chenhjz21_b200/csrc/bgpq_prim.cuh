@@ -71,7 +71,9 @@ __device__ __forceinline__ void fence_proxy_async() {
 // Node lock (D4): test-and-test-and-set with an acquire CAS; one elected thread spins
 // with __nanosleep backoff so the CAS traffic does not starve the holder's accesses.
 __device__ __forceinline__ u32 lock_acquire(u32* lk) {
-  u32 spins = 0, ns = 16;
+  if (cas_acquire(lk, 0u, 1u) == 0u) return 0;  // uncontended: one round trip
+  u32 spins = 1, ns = 16;
+  __nanosleep(ns);
   for (;;) {
     if (ld_relaxed(lk) == 0u && cas_acquire(lk, 0u, 1u) == 0u) return spins;
     ++spins;
@@ -83,6 +85,14 @@ __device__ __forceinline__ u32 lock_acquire(u32* lk) {
 // this thread with a CTA barrier (bar.sync is morally strong and orders them before this
 // thread's later accesses); the gpu-scope release store is cumulative and publishes them.
 __device__ __forceinline__ void lock_release(u32* lk) { st_release(lk, 0u); }
+
+// The cached {state, min, max} of a node's 16-B metadata record, in one load (several of
+// these issue back to back; a separate relaxed load per word would serialise on their uses).
+__device__ __forceinline__ void meta_load(const void* rec, u32& st, u32& mn, u32& mx) {
+  u32 lk;
+  asm volatile("ld.relaxed.gpu.global.v4.u32 {%0, %1, %2, %3}, [%4];"
+               : "=r"(lk), "=r"(st), "=r"(mn), "=r"(mx) : "l"(rec) : "memory");
+}
 
 // mbarrier + TMA bulk copy (global -> shared), completion by transaction bytes.
 __device__ __forceinline__ void mbar_init(u64* bar, u32 count) {
