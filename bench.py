@@ -338,9 +338,12 @@ def measure_mix(args, world, rank, local, dist, q_factory=None):
                                 f"keys, K={K}, w={w} B; keys/s = (in + out)/2/t") if P else
                    (f"C2 mix: empty heap, {n_pairs} insert(K) + {n_pairs} deletemin(K) pairs"),
                    "n_keys": n, "K": K, "w_bytes": w, "prefill": P, "dist": args.dist,
-                   "execution": "bgpq_run_mixed: persistent CTAs, per-node locks + lock warp (bgpq_locks_kernel)",
+                   "execution": ("bgpq_run_mixed: the leading (INSERT(K), DELETEMIN(K)) pairs on the cluster "
+                                 "engine (bgpq_msort_kernel sorts the batches, bgpq_dsys_kernel runs each pair "
+                                 "as the MARKED hand-off at the root, reading R26), the rest of the call on the "
+                                 "per-node-lock engine (bgpq_locks_kernel)"),
                    "l2": "heap and inputs larger than the 126 MB L2; no flush"},
-        "roofline": {"bound": "hbm", "kernel": "bgpq_locks_kernel (the mixed call)", "achieved": achieved,
+        "roofline": {"bound": "hbm", "kernel": "bgpq_dsys_kernel (the mixed call's pairs)", "achieved": achieved,
                      "peak": peak, "unit": "GB/s", "frac": achieved / peak, "traffic": None,
                      "peak_source": peak_src, "alg_bytes_per_launch": bm["total"]},
         "counters_per_step": dst, "gpu_launches": launches,
