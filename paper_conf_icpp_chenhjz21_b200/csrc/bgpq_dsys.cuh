@@ -96,6 +96,7 @@ struct DsCtl {
   u32 ns[DS_MAXOWN], mn[DS_MAXOWN], mx[DS_MAXOWN], pend[DS_MAXOWN];
   ull st[NSTAT];
   ull tm[8];  // debug timers (bgpq_set_debug bit 1024): total, wait-above, wait-children, split, wait-b, sends
+  ull tm2[16];  // debug 2097152: R1's per-segment timers (tools/ds_seg.py)
 };
 constexpr size_t DSCTL_BYTES = (sizeof(DsCtl) + 127) / 128 * 128;
 
@@ -176,6 +177,11 @@ struct DsRole {
   u32 lph;                // lbar parity
   bool timing;
   __device__ __forceinline__ ull tnow() const { return timing ? clock64() : 0ull; }
+  bool seg = false;  // debug 2097152: segment timers of R1
+  ull tseg = 0;
+  __device__ __forceinline__ void segmark(int k) {
+    if (seg) { const ull t = clock64(); c->tm2[k] += t - tseg; tseg = t; }
+  }
   __device__ __forceinline__ void tacc(int k, ull t0) { if (timing) c->tm[k] += clock64() - t0; }
 
   __device__ __forceinline__ u32* BK(u32 s) const { return sk + s * K; }
@@ -768,10 +774,13 @@ __device__ void ds_level(DsRole<K, V>& R, const u64 m) {
   u32 push_old = DS_NONE;  // slot whose push may still be reading it
   u32 a_src = 0, a_cmin = 0, a_cmax = 0, early = 0;  // thread 0: the path message's refill-key info
   const ull t_start = R.tnow();
+  if (tid == 0) R.tseg = clock64();
   for (u64 i = 0; i < m; ++i) {
     if (tid == 0) {
       const ull t1 = R.tnow();
+      R.segmark(15);
       const DsMsg a = R.recv();
+      R.segmark(0);
       R.tacc(1, t1);
       c->b[0] = 0;
       if (a.kind == MK_ASTOP) {  // the walk stopped above: nothing at this depth
@@ -790,6 +799,7 @@ __device__ void ds_level(DsRole<K, V>& R, const u64 m) {
           }
         }
         R.tacc(2, t2);
+        R.segmark(1);
         const u32 x = mx[jl] > mx[jr] ? l : r, y = l + r - x;  // l.9 (R6)
         const u32 minc = mn[jl] < mn[jr] ? mn[jl] : mn[jr];
         // early commit (MA_EARLY): the carried keys are R = [a.cmin, a.cmax] at a.src if every
@@ -804,14 +814,17 @@ __device__ void ds_level(DsRole<K, V>& R, const u64 m) {
         c->b[7] = sy; c->b[9] = a.slot;
         c->b[10] = (mx[jl] <= mn[jr] || mx[jr] <= mn[jl]) ? 1u : 0u;
         c->b[13] = minc;
+        R.segmark(2);
       }
     }
     cta_bar<DS_NT>();
+    if (tid == 0) R.segmark(3);
     if (c->b[0]) continue;
     const u32 sl = c->b[1], sr = c->b[2], A = c->b[3], B = c->b[4];
     const ull t3 = R.tnow();
     ds_split<K, V>(R, sl, sr, A, B);  // l.10 (speculative until message b)
     if (tid == 0) {
+      R.segmark(4);
       R.tacc(3, t3);
       const u32 x = c->b[5], y = c->b[6], sy = c->b[7], up = c->b[9];
       const u32 minc = c->b[13];
@@ -830,11 +843,15 @@ __device__ void ds_level(DsRole<K, V>& R, const u64 m) {
         R.release(sl); R.release(sr);
         ns[jx] = B; mn[jx] = R.BK(B)[0]; mx[jx] = R.BK(B)[K - 1];
         ns[jy] = sy; pend[jy] = 1;
+        R.segmark(5);
         R.push_up(A, up);
+        R.segmark(6);
         push_old = A;
         R.send((u32)i, MK_B, 0, 0, a_src, a_cmin, a_cmax);
+        R.segmark(7);
         const ull t4 = R.tnow();
         const DsMsg b = R.recv();  // the level above's message b, consumed in order
+        R.segmark(8);
         R.tacc(4, t4);
         if (b.kind != MK_B || b.src != a_src) __trap();  // contradicts the argument above
       } else {
@@ -880,6 +897,7 @@ __device__ void ds_level(DsRole<K, V>& R, const u64 m) {
       }
     }
     cta_bar<DS_NT>();
+    if (tid == 0) R.segmark(9);
     if (c->b[14]) {  // rare: a real (cur, y) merge at this depth
       const u32 cs = c->b[4], lo = c->b[5], hi = c->b[6], Y = c->b[12];
       ds_split<K, V>(R, cs, Y, lo, hi);
@@ -1150,6 +1168,7 @@ __global__ void __cluster_dims__(DS_CL, 1, 1) __launch_bounds__(DS_BLOCK, 1)
     R.fm = (R.rank == DS_CL - 1) ? ((1u << (DS_NSLOT - 8)) - 1u) : ((1u << DS_NSLOT) - 1u);
     R.sbph = 0; R.in_seq = 0; R.out_seq = 0; R.out_seq2 = 0; R.lph = 0;
     R.timing = (C.debug & 1024u) != 0;
+    R.seg = (C.debug & 2097152u) != 0 && cl_rank() == 1;
     if (threadIdx.x == 0) {
       for (u32 e = 0; e < DS_RING; ++e) mbar_init(&c->inbar[e], 1);
       for (u32 e = 0; e < DS_RING; ++e) R.arm_inbox(e);
@@ -1165,6 +1184,7 @@ __global__ void __cluster_dims__(DS_CL, 1, 1) __launch_bounds__(DS_BLOCK, 1)
       }
       for (int q = 0; q < NSTAT; ++q) c->st[q] = 0;
       for (int q = 0; q < 8; ++q) c->tm[q] = 0;
+      for (int q = 0; q < 16; ++q) c->tm2[q] = 0;
       asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     __syncthreads();
@@ -1199,6 +1219,10 @@ __global__ void __cluster_dims__(DS_CL, 1, 1) __launch_bounds__(DS_BLOCK, 1)
       if (R.timing) {
         ull* tms = reinterpret_cast<ull*>(H.hdr + H_TIME);
         for (int q = 0; q < 6; ++q) atomicAdd(tms + 6 * R.rank + q, c->tm[q]);
+      }
+      if (R.seg) {
+        ull* tms = reinterpret_cast<ull*>(H.hdr + H_TIME);
+        for (int q = 0; q < 16; ++q) atomicAdd(tms + q, c->tm2[q]);
       }
     }
     cluster_sync_all();  // no CTA leaves while a peer may still access its shared memory
