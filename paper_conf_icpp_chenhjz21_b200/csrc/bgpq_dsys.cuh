@@ -45,6 +45,7 @@ constexpr u32 DS_CREDIT = 4;           // credits are returned every DS_CREDIT e
 constexpr u32 DS_RF = 8;               // refill takes run at most this many ops ahead (R20)
 constexpr u32 DS_HMIN = 1024;          // heapSize floor of the engine (depth >= 10 > DS_RF)
 constexpr u32 DS_NONE = 0xFFFFFFFFu;
+constexpr u32 DS_PULL = 0x40000000u;   // carried-keys source: a slot in a role's shared memory
 constexpr u32 DSM_HMIN = 64;           // mixed calls: heapSize floor (nodes 1..63 AVAIL: the levels
                                        // and the stager's children are never EMPTY)
 
@@ -83,6 +84,7 @@ struct DsCtl {
   u32 rf_min[DS_RF], rf_max[DS_RF];
   u32 rf_used;           // ops whose take thread 0 consumed
   u32 pfs[4];            // mixed calls: R0's prefetch ring of sorted INSERT batches (slots)
+  u32 pfreed;            // slots holding carried keys a lower level has pulled (remote red.or)
   // stager: helper A (LOCK + stage children) and helper B (tasks, write-backs, UNLOCKs) rings
   u32 sq_done;           // staging records published (helper A -> thread 0), one per op
   u32 sq_ret;            // ops whose staging slots thread 0 returned
@@ -186,8 +188,46 @@ struct DsRole {
 
   __device__ __forceinline__ u32* BK(u32 s) const { return sk + s * K; }
   __device__ __forceinline__ u32* BV(u32 s) const { return V ? sv + s * K : nullptr; }
+  // ---- carried keys that live only in a role's shared memory (a (cur, y) SORT_SPLIT merged
+  // them on chip): message b names them as PULL | owner rank << 8 | slot; the level that needs
+  // their content copies them over DSMEM (pull_copy) and returns the slot (pull_free).
+  __device__ __forceinline__ u32 pull_ref(u32 s) const { return DS_PULL | (rank << 8) | s; }
+  // thread 0, before the message b that carries a pull reference: the compute threads' writes
+  // of the slot (ordered before thread 0 by the CTA barrier) are released at cluster scope
+  __device__ __forceinline__ void pull_publish() const { asm volatile("fence.acq_rel.cluster;" ::: "memory"); }
+  // all DS_NT compute threads (the caller's thread 0 ran fence.acq_rel.cluster after the
+  // message and a CTA barrier followed): slot `dst` <- the referenced slot of its owner
+  __device__ __forceinline__ void pull_copy(u32 ref, u32 dst) const {
+    const u32 owner = (ref >> 8) & 0xFFu, src = ref & 0xFFu;
+    const u32 rk = cl_map(BK(src), owner);
+    for (int q = threadIdx.x; q < K / 4; q += DS_NT) {
+      uint4 v;
+      asm volatile("ld.shared::cluster.v4.u32 {%0, %1, %2, %3}, [%4];"
+                   : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(rk + 16u * q) : "memory");
+      reinterpret_cast<uint4*>(BK(dst))[q] = v;
+    }
+    if (V) {
+      const u32 rv = cl_map(BV(src), owner);
+      for (int q = threadIdx.x; q < K / 4; q += DS_NT) {
+        uint4 v;
+        asm volatile("ld.shared::cluster.v4.u32 {%0, %1, %2, %3}, [%4];"
+                     : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(rv + 16u * q) : "memory");
+        reinterpret_cast<uint4*>(BV(dst))[q] = v;
+      }
+    }
+  }
+  // thread 0, after the CTA barrier that ended pull_copy: the owner may reuse the slot
+  __device__ __forceinline__ void pull_free(u32 ref) const {
+    const u32 owner = (ref >> 8) & 0xFFu, src = ref & 0xFFu;
+    asm volatile("red.relaxed.cluster.shared::cluster.or.b32 [%0], %1;" ::"r"(cl_map(&c->pfreed, owner)),
+                 "r"(1u << src) : "memory");
+  }
+  __device__ __forceinline__ void collect_pulled() { fm |= atomicExch(&c->pfreed, 0u); }
   __device__ __forceinline__ u32 alloc() {
-    if (fm == 0) __trap();
+    while (fm == 0) {  // slots lent to lower levels for pulls come back through pfreed
+      const u32 fr = atomicExch(&c->pfreed, 0u);
+      fm |= fr;
+    }
     const u32 s = __ffs(fm) - 1;
     fm &= ~(1u << s);
     return s;
@@ -371,6 +411,7 @@ __device__ void ds_r0(DsRole<K, V>& R, const u64 m) {
   const ull t_start = R.tnow();
   for (u64 i = 0; i < m; ++i) {
     if (tid == 0) {
+      R.collect_pulled();
       // refill of op i (Alg.2 l.5-12), taken ahead by the helper: node hs, now EMPTY
       const u32 t = hs;
       const ull t1 = R.tnow();
@@ -443,13 +484,12 @@ __device__ void ds_r0(DsRole<K, V>& R, const u64 m) {
       const u32 r = c->b[11], lo = c->b[12], hi = c->b[13];
       ds_split<K, V>(R, r, A, lo, hi);
       if (tid == 0) {
-        const u32 y = c->b[6];
-        R.store_node(y, hi);  // C1 in y1's HBM copy (y1 is on chip; its HBM copy is dead)
-        __threadfence();
-        R.send((u32)i, MK_B, 0, 0, y, R.BK(hi)[0], R.BK(hi)[K - 1]);
+        // C1 stays in slot hi; the level that needs its content pulls it (DS_PULL)
+        R.pull_publish();
+        R.send((u32)i, MK_B, 0, 0, R.pull_ref(hi), R.BK(hi)[0], R.BK(hi)[K - 1]);
         if (rz) output(i, lo);
         else { ns[1] = lo; mn[1] = R.BK(lo)[0]; mx[1] = R.BK(lo)[K - 1]; }
-        R.release(r); R.release(hi); R.release(A);
+        R.release(r); R.release(A);
       }
       cta_bar<DS_NT>();
     }
@@ -555,6 +595,7 @@ __device__ void ds_r0_mixed(DsRole<K, V>& R, const u64 m) {
     const u64 jd = 2 * i + 1;  // the DELETEMIN's op index (the INSERT is 2i)
     // ---- INSERT, Alg.1 l.20: (root, items) <- SORT_SPLIT(root, |root|, items, K, |root|)
     if (tid == 0) {
+      R.collect_pulled();
       if (i + PF < m) prefetch(i + PF);
       const ull t1 = R.tnow();
       mbar_wait(&c->sbar[i % 4], (pfph >> (i % 4)) & 1u);
@@ -564,13 +605,12 @@ __device__ void ds_r0_mixed(DsRole<K, V>& R, const u64 m) {
       imin = R.BK(it)[0];
       imax = R.BK(it)[K - 1];
       const ull t2 = R.tnow();
-      for (u32 q = 2; q <= 3; ++q)  // op i-1's y1 push must have landed (depth 1 is read below)
-        if (pend[q]) {
-          R.wait_pushed(ns[q]);
-          pend[q] = 0;
-          mn[q] = R.BK(ns[q])[0];
-          mx[q] = R.BK(ns[q])[K - 1];
-        }
+      if (pend[d1]) {  // the INSERT's depth-1 node: op i-1's push into it must have landed
+        R.wait_pushed(ns[d1]);
+        pend[d1] = 0;
+        mn[d1] = R.BK(ns[d1])[0];
+        mx[d1] = R.BK(ns[d1])[K - 1];
+      }
       R.tacc(2, t2);
       c->st[S_INS_OPS]++;
       c->st[S_INS_HEAPIFY]++;
@@ -619,6 +659,15 @@ __device__ void ds_r0_mixed(DsRole<K, V>& R, const u64 m) {
     // ---- DELETEMIN: the root's keys are its output (Alg.2 l.22), the refill keys are the
     // INSERT's items (the MARKED hand-off, l.7-12), then Alg.3 at the root as in ds_r0
     if (tid == 0) {
+      const u32 o1 = 5u - d1;  // the other depth-1 node, read by the depth-0 step only
+      if (pend[o1]) {
+        const ull t2 = R.tnow();
+        R.wait_pushed(ns[o1]);
+        pend[o1] = 0;
+        mn[o1] = R.BK(ns[o1])[0];
+        mx[o1] = R.BK(ns[o1])[K - 1];
+        R.tacc(2, t2);
+      }
       c->st[S_DEL_OPS]++;
       c->st[S_DEL_REFILL]++;
       c->st[S_MARKED]++;
@@ -659,16 +708,13 @@ __device__ void ds_r0_mixed(DsRole<K, V>& R, const u64 m) {
       const u32 ymax = R.BK(A)[K - 1];
       if (ymax <= imin) {  // l.12 is a swap: root <- Y, the refill keys sink on (by reference)
         c->st[S_DEL_CY_SWAP]++;
-        if (dirty) {  // the items changed on chip: H.xk + i*K must hold them before the reference
-          asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-          bulk_s2g(H.xk + (size_t)i * K, R.BK(it), NB);
-          if (V) bulk_s2g(H.xv + (size_t)i * K, R.BV(it), NB);
-          asm volatile("cp.async.bulk.commit_group;" ::: "memory");
-          asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
-          __threadfence();
+        if (dirty) {  // the items changed on chip: a lower level pulls them from slot it
+          R.pull_publish();
+          R.send((u32)i, MK_B, 0, 0, R.pull_ref(it), imin, imax);
+        } else {      // still the sorted batch H.xk + i*K
+          R.send((u32)i, MK_B, 0, 0, XREF | (u32)i, imin, imax);
+          R.release(it);
         }
-        R.send((u32)i, MK_B, 0, 0, XREF | (u32)i, imin, imax);
-        R.release(it);
         if (rz) output(jd, A);
         else { ns[1] = A; mn[1] = R.BK(A)[0]; mx[1] = ymax; }
         c->b[15] = 0;
@@ -684,13 +730,11 @@ __device__ void ds_r0_mixed(DsRole<K, V>& R, const u64 m) {
       const u32 r = c->b[11], lo = c->b[12], hi = c->b[13];
       ds_split<K, V>(R, r, A, lo, hi);
       if (tid == 0) {
-        const u32 y = c->b[6];
-        R.store_node(y, hi);
-        __threadfence();
-        R.send((u32)i, MK_B, 0, 0, y, R.BK(hi)[0], R.BK(hi)[K - 1]);
+        R.pull_publish();  // C1 stays in slot hi until a lower level pulled it
+        R.send((u32)i, MK_B, 0, 0, R.pull_ref(hi), R.BK(hi)[0], R.BK(hi)[K - 1]);
         if (rz) output(jd, lo);
         else { ns[1] = lo; mn[1] = R.BK(lo)[0]; mx[1] = R.BK(lo)[K - 1]; }
-        R.release(r); R.release(hi); R.release(A);
+        R.release(r); R.release(A);
       }
       cta_bar<DS_NT>();
     }
@@ -777,6 +821,7 @@ __device__ void ds_level(DsRole<K, V>& R, const u64 m) {
   if (tid == 0) R.tseg = clock64();
   for (u64 i = 0; i < m; ++i) {
     if (tid == 0) {
+      R.collect_pulled();
       const ull t1 = R.tnow();
       R.segmark(15);
       const DsMsg a = R.recv();
@@ -868,9 +913,14 @@ __device__ void ds_level(DsRole<K, V>& R, const u64 m) {
         R.send((u32)i, MK_BSTOP);
       } else if (b.cmax <= minc) {  // l.4: stop at cur — cur keeps the carried keys
         const u32 s = R.alloc();
-        R.load_node(s, b.src);
-        R.push_up(s, up);
-        push_old = s;
+        if (b.src & DS_PULL) {  // on chip above: pulled by all threads below, then pushed up
+          asm volatile("fence.acq_rel.cluster;" ::: "memory");
+          c->b[14] = 2; c->b[4] = s; c->b[9] = up; c->b[15] = b.src;
+        } else {
+          R.load_node(s, b.src);
+          R.push_up(s, up);
+          push_old = s;
+        }
         R.release(A); R.release(B);
         R.disarm_slot(sy);
         R.release(sy);
@@ -888,28 +938,39 @@ __device__ void ds_level(DsRole<K, V>& R, const u64 m) {
           R.push_up(A, up);
           push_old = A;
           R.send((u32)i, MK_B, 0, 0, b.src, b.cmin, b.cmax);
-        } else {  // l.12 merges: (cur, C) <- SORT_SPLIT(carried, Y); C into y's dead HBM copy
+        } else {  // l.12 merges: (cur, C) <- SORT_SPLIT(carried, Y); C stays on chip (DS_PULL)
           const u32 cs = R.alloc(), lo = R.alloc(), hi = R.alloc();
-          R.load_node(cs, b.src);
+          if (b.src & DS_PULL) asm volatile("fence.acq_rel.cluster;" ::: "memory");
+          else R.load_node(cs, b.src);
           c->b[14] = 1; c->b[4] = cs; c->b[5] = lo; c->b[6] = hi; c->b[7] = y; c->b[9] = up; c->b[12] = A;
+          c->b[15] = b.src;
         }
       }
       }
     }
     cta_bar<DS_NT>();
     if (tid == 0) R.segmark(9);
-    if (c->b[14]) {  // rare: a real (cur, y) merge at this depth
-      const u32 cs = c->b[4], lo = c->b[5], hi = c->b[6], Y = c->b[12];
-      ds_split<K, V>(R, cs, Y, lo, hi);
+    if (c->b[14] == 2) {  // stop at cur with carried keys on chip above: pull, push up
+      const u32 s2 = c->b[4], up = c->b[9], ref = c->b[15];
+      R.pull_copy(ref, s2);
+      cta_bar<DS_NT>();
       if (tid == 0) {
-        const u32 y = c->b[7], up = c->b[9];
-        R.store_node(y, hi);  // the new carried keys in y's HBM copy
-        __threadfence();
+        R.pull_free(ref);
+        R.push_up(s2, up);
+        push_old = s2;
+      }
+    } else if (c->b[14]) {  // a real (cur, y) merge at this depth
+      const u32 cs = c->b[4], lo = c->b[5], hi = c->b[6], Y = c->b[12], ref = c->b[15];
+      if (ref & DS_PULL) R.pull_copy(ref, cs);
+      ds_split<K, V>(R, cs, Y, lo, hi);  // (begins with a CTA barrier)
+      if (tid == 0) {
+        if (ref & DS_PULL) R.pull_free(ref);
+        const u32 up = c->b[9];
         R.push_up(lo, up);
         push_old = lo;
         R.release(cs); R.release(Y);
-        R.send((u32)i, MK_B, 0, 0, y, R.BK(hi)[0], R.BK(hi)[K - 1]);
-        R.release(hi);
+        R.pull_publish();  // the new carried keys stay in slot hi until a lower level pulled them
+        R.send((u32)i, MK_B, 0, 0, R.pull_ref(hi), R.BK(hi)[0], R.BK(hi)[K - 1]);
       }
       cta_bar<DS_NT>();
     }
@@ -1003,9 +1064,14 @@ __device__ void ds_stager(DsRole<K, V>& R, const u64 m) {
       if (b.kind == MK_BSTOP || b.cmax <= minc) {  // stopped above / at cur: nothing changes below
         if (b.kind != MK_BSTOP) {                  // cur keeps the carried keys
           const u32 s = R.alloc();
-          R.load_node(s, b.src);
-          R.push_up(s, up);
-          push_old = s;
+          if (b.src & DS_PULL) {
+            asm volatile("fence.acq_rel.cluster;" ::: "memory");
+            c->b[14] = 2; c->b[4] = s; c->b[9] = up; c->b[15] = b.src;
+          } else {
+            R.load_node(s, b.src);
+            R.push_up(s, up);
+            push_old = s;
+          }
         }
         sq_req<K, V>(R, &c->wq_head, &c->wq_done, c->wq, WQ_CANCEL, y, l, r, 0);
         R.release(A); R.release(B);
@@ -1021,19 +1087,46 @@ __device__ void ds_stager(DsRole<K, V>& R, const u64 m) {
           c->st[S_DEL_CY_SWAP]++;
           R.push_up(A, up);
           push_old = A;
-          sq_req<K, V>(R, &c->wq_head, &c->wq_done, c->wq, WQ_COMMIT, y, b.src, 0, 0);
+          if (b.src & DS_PULL) {  // on chip above: pull them and store them in y's HBM copy
+            asm volatile("fence.acq_rel.cluster;" ::: "memory");
+            c->b[14] = 3; c->b[4] = R.alloc(); c->b[7] = y; c->b[15] = b.src;
+          } else {
+            sq_req<K, V>(R, &c->wq_head, &c->wq_done, c->wq, WQ_COMMIT, y, b.src, 0, 0);
+          }
         } else {
           const u32 cs = R.alloc(), lo = R.alloc(), hi = R.alloc();
-          R.load_node(cs, b.src);
+          if (b.src & DS_PULL) asm volatile("fence.acq_rel.cluster;" ::: "memory");
+          else R.load_node(cs, b.src);
           c->b[14] = 1; c->b[4] = cs; c->b[5] = lo; c->b[6] = hi; c->b[7] = y; c->b[9] = up; c->b[12] = A;
+          c->b[15] = b.src;
         }
       }
     }
     cta_bar<DS_NT>();
-    if (c->b[14]) {  // rare: a real (cur, y) merge
-      const u32 cs = c->b[4], lo = c->b[5], hi = c->b[6], Y = c->b[12];
+    if (c->b[14] == 2 || c->b[14] == 3) {  // carried keys on chip above: pull them
+      const u32 s2 = c->b[4], ref = c->b[15], mode = c->b[14];
+      R.pull_copy(ref, s2);
+      cta_bar<DS_NT>();
+      if (tid == 0) {
+        R.pull_free(ref);
+        if (mode == 2) {  // stop at cur: cur <- the carried keys
+          R.push_up(s2, c->b[9]);
+          push_old = s2;
+        } else {  // swap: the walker below y reads them from y's HBM copy (y is LOCKed by us)
+          const u32 y = c->b[7];
+          R.store_node(y, s2);
+          __threadfence();
+          R.release(s2);
+          sq_req<K, V>(R, &c->wq_head, &c->wq_done, c->wq, WQ_COMMIT, y, y, 0, 0);
+        }
+      }
+      cta_bar<DS_NT>();
+    } else if (c->b[14]) {  // a real (cur, y) merge
+      const u32 cs = c->b[4], lo = c->b[5], hi = c->b[6], Y = c->b[12], ref = c->b[15];
+      if (ref & DS_PULL) R.pull_copy(ref, cs);
       ds_split<K, V>(R, cs, Y, lo, hi);
       if (tid == 0) {
+        if (ref & DS_PULL) R.pull_free(ref);
         const u32 y = c->b[7], up = c->b[9];
         R.store_node(y, hi);  // the carried keys in y's HBM copy (y is LOCKed by us)
         __threadfence();
@@ -1176,7 +1269,7 @@ __global__ void __cluster_dims__(DS_CL, 1, 1) __launch_bounds__(DS_BLOCK, 1)
       mbar_init(&c->lbar, 1);
       mbar_init(&c->hbar, 1);
       for (int q = 0; q < 4; ++q) mbar_init(&c->sbar[q], 1);
-      c->consumed = 0; c->rf_seq = 0; c->rf_used = 0; c->tasks = 0; c->quit = 0;
+      c->consumed = 0; c->rf_seq = 0; c->rf_used = 0; c->tasks = 0; c->quit = 0; c->pfreed = 0;
       c->sq_done = 0; c->sq_ret = 0; c->wq_head = 0; c->wq_done = 0; c->wb_free = 0; c->aconsumed = 0;
       for (u32 e = 0; e < DS_RING; ++e) {
         mbar_init(&c->ainbar[e], 1);
