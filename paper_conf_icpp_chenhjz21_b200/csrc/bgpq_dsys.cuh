@@ -178,6 +178,19 @@ struct DsRole {
   u32 out_seq2;           // path messages sent to the stager's second inbox
   u32 lph;                // lbar parity
   bool timing;
+  // thread 0's per-op counters in registers (a shared-memory u64 read-modify-write per counter
+  // per op sat on the decision chain); flushed into c->st by flush_counts at the role's end
+  u32 n_lev = 0, n_nomove = 0, n_swap = 0, n_ilev = 0, n_inoop = 0, n_iswap = 0;
+  __device__ __forceinline__ void flush_counts() {
+    c->st[S_DEL_LEVELS] += n_lev;
+    c->st[S_DEL_LR_NOMOVE] += n_nomove;
+    c->st[S_DEL_LR_MERGE] += n_lev - n_nomove;
+    c->st[S_DEL_CY_SWAP] += n_swap;
+    c->st[S_INS_LEVELS] += n_ilev;
+    c->st[S_INS_NOOP] += n_inoop;
+    c->st[S_INS_SWAP] += n_iswap;
+    c->st[S_INS_MERGE] += n_ilev - n_inoop - n_iswap;
+  }
   __device__ __forceinline__ ull tnow() const { return timing ? clock64() : 0ull; }
   bool seg = false;  // debug 2097152: segment timers of R1
   ull tseg = 0;
@@ -431,8 +444,6 @@ __device__ void ds_r0(DsRole<K, V>& R, const u64 m) {
         }
       R.tacc(2, t2);
       if (!rz) output(i, ns[1]);  // Alg.2 l.22: the root's K keys are op i's output
-      c->st[S_DEL_OPS]++;
-      c->st[S_DEL_REFILL]++;
       // Alg.3 at the root: cur = root holding the refill keys
       const u32 minc = mn[2] < mn[3] ? mn[2] : mn[3];
       if (rmax <= minc) {  // l.4: stop at the root — root <- the refill keys
@@ -450,8 +461,8 @@ __device__ void ds_r0(DsRole<K, V>& R, const u64 m) {
         const u32 A = R.alloc(), B = R.alloc();
         c->b[0] = 0; c->b[1] = ns[2]; c->b[2] = ns[3]; c->b[3] = A; c->b[4] = B;
         c->b[5] = x; c->b[6] = y; c->b[7] = sy; c->b[8] = t; c->b[9] = rmin; c->b[10] = rmax;
-        c->st[S_DEL_LEVELS]++;
-        c->st[(mx[2] <= mn[3] || mx[3] <= mn[2]) ? S_DEL_LR_NOMOVE : S_DEL_LR_MERGE]++;
+        ++R.n_lev;
+        R.n_nomove += (mx[2] <= mn[3] || mx[3] <= mn[2]) ? 1u : 0u;
       }
     }
     cta_bar<DS_NT>();
@@ -465,7 +476,7 @@ __device__ void ds_r0(DsRole<K, V>& R, const u64 m) {
       R.release(s2); R.release(s3);
       const u32 ymax = R.BK(A)[K - 1];
       if (ymax <= rmin) {  // l.12 is a swap: root <- Y, the refill keys sink on (by reference)
-        c->st[S_DEL_CY_SWAP]++;
+        ++R.n_swap;
         R.send((u32)i, MK_B, 0, 0, t, rmin, rmax);
         if (rz) output(i, A);  // Alg.3 l.5-6 / l.13: the root's new keys are extracted
         else { ns[1] = A; mn[1] = R.BK(A)[0]; mx[1] = ymax; }
@@ -510,6 +521,9 @@ __device__ void ds_r0(DsRole<K, V>& R, const u64 m) {
     asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(lin) : "l"(H.hdr + H_LIN) : "memory");
     asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(H.hdr + H_LIN), "l"(lin + m) : "memory");
     c->st[S_KEYS_OUT] += m * (u64)K;
+    c->st[S_DEL_OPS] += m;
+    c->st[S_DEL_REFILL] += m;
+    R.flush_counts();
     if (R.C.d_count && m) atomicAdd(R.C.d_count, (ull)(m * (u64)K));
     *reinterpret_cast<volatile u64*>(R.D.op_base) = m;
   }
@@ -612,8 +626,7 @@ __device__ void ds_r0_mixed(DsRole<K, V>& R, const u64 m) {
         mx[d1] = R.BK(ns[d1])[K - 1];
       }
       R.tacc(2, t2);
-      c->st[S_INS_OPS]++;
-      c->st[S_INS_HEAPIFY]++;
+
       const u32 ra = rz ? 0u : (mx[1] <= imin) ? 0u : (imax <= mn[1]) ? 1u : 2u;
       if (ra == 1) {  // the batch lies entirely below the root: swap the contents
         const u32 t = ns[1]; ns[1] = it; it = t;
@@ -636,8 +649,9 @@ __device__ void ds_r0_mixed(DsRole<K, V>& R, const u64 m) {
     // ---- INSERT, l.33 at cur = NEXT(root, tar): (Heap[cur], items) <- SORT_SPLIT(Heap[cur], items)
     if (tid == 0) {
       const u32 da = (mx[d1] <= imin) ? 0u : (imax <= mn[d1]) ? 1u : 2u;
-      c->st[S_INS_LEVELS]++;
-      c->st[da == 0 ? S_INS_NOOP : da == 1 ? S_INS_SWAP : S_INS_MERGE]++;
+      ++R.n_ilev;
+      R.n_inoop += da == 0 ? 1u : 0u;
+      R.n_iswap += da == 1 ? 1u : 0u;
       if (da == 1) {
         const u32 t = ns[d1]; ns[d1] = it; it = t;
         const u32 a = mn[d1], b = mx[d1]; mn[d1] = imin; mx[d1] = imax; imin = a; imax = b;
@@ -668,9 +682,7 @@ __device__ void ds_r0_mixed(DsRole<K, V>& R, const u64 m) {
         mx[o1] = R.BK(ns[o1])[K - 1];
         R.tacc(2, t2);
       }
-      c->st[S_DEL_OPS]++;
-      c->st[S_DEL_REFILL]++;
-      c->st[S_MARKED]++;
+
       if (C.lin_ticket) {
         st_relaxed_u64(reinterpret_cast<u64*>(C.lin_ticket) + 2 * i, lin0 + 2 * i);
         st_relaxed_u64(reinterpret_cast<u64*>(C.lin_ticket) + jd, lin0 + jd);
@@ -692,8 +704,8 @@ __device__ void ds_r0_mixed(DsRole<K, V>& R, const u64 m) {
         const u32 A = R.alloc(), B = R.alloc();
         c->b[0] = 0; c->b[1] = ns[2]; c->b[2] = ns[3]; c->b[3] = A; c->b[4] = B;
         c->b[5] = x; c->b[6] = y; c->b[7] = sy;
-        c->st[S_DEL_LEVELS]++;
-        c->st[(mx[2] <= mn[3] || mx[3] <= mn[2]) ? S_DEL_LR_NOMOVE : S_DEL_LR_MERGE]++;
+        ++R.n_lev;
+        R.n_nomove += (mx[2] <= mn[3] || mx[3] <= mn[2]) ? 1u : 0u;
       }
     }
     cta_bar<DS_NT>();
@@ -707,7 +719,7 @@ __device__ void ds_r0_mixed(DsRole<K, V>& R, const u64 m) {
       R.release(s2); R.release(s3);
       const u32 ymax = R.BK(A)[K - 1];
       if (ymax <= imin) {  // l.12 is a swap: root <- Y, the refill keys sink on (by reference)
-        c->st[S_DEL_CY_SWAP]++;
+        ++R.n_swap;
         if (dirty) {  // the items changed on chip: a lower level pulls them from slot it
           R.pull_publish();
           R.send((u32)i, MK_B, 0, 0, R.pull_ref(it), imin, imax);
@@ -753,6 +765,12 @@ __device__ void ds_r0_mixed(DsRole<K, V>& R, const u64 m) {
     asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(H.hdr + H_LIN), "l"(lin0 + 2 * m) : "memory");
     st_relaxed(H.hdr + H_FETCH, (u32)(2 * m));  // the lock engine continues at op 2m
     c->st[S_KEYS_OUT] += m * (u64)K;
+    c->st[S_INS_OPS] += m;
+    c->st[S_INS_HEAPIFY] += m;
+    c->st[S_DEL_OPS] += m;
+    c->st[S_DEL_REFILL] += m;
+    c->st[S_MARKED] += m;
+    R.flush_counts();
     *reinterpret_cast<volatile u64*>(R.D.op_base) = m;
   }
 }
@@ -879,18 +897,19 @@ __device__ void ds_level(DsRole<K, V>& R, const u64 m) {
         // (max(Y_k) <= max(y_k+1) <= min(children of y_k+1) <= max(Y_k+1), heap order), so every
         // (cur, y) split above was a swap passing R on unchanged, and so is this one: cur <- Y
         // is final now (pushed up before the level above's message b arrives), R sinks on.
-        asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+        // The push goes first: the level above is waiting for it.
+        R.segmark(5);
+        R.push_up(A, up);
+        R.segmark(6);
+        asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");  // all but this push read
         R.release(push_old);
-        c->st[S_DEL_LEVELS]++;
-        c->st[c->b[10] ? S_DEL_LR_NOMOVE : S_DEL_LR_MERGE]++;
-        c->st[S_DEL_CY_SWAP]++;
+        ++R.n_lev;
+        R.n_nomove += c->b[10];
+        ++R.n_swap;
         const u32 jx = x - base, jy = y - base;
         R.release(sl); R.release(sr);
         ns[jx] = B; mn[jx] = R.BK(B)[0]; mx[jx] = R.BK(B)[K - 1];
         ns[jy] = sy; pend[jy] = 1;
-        R.segmark(5);
-        R.push_up(A, up);
-        R.segmark(6);
         push_old = A;
         R.send((u32)i, MK_B, 0, 0, a_src, a_cmin, a_cmax);
         R.segmark(7);
@@ -926,15 +945,15 @@ __device__ void ds_level(DsRole<K, V>& R, const u64 m) {
         R.release(sy);
         R.send((u32)i, MK_BSTOP);
       } else {
-        c->st[S_DEL_LEVELS]++;
-        c->st[c->b[10] ? S_DEL_LR_NOMOVE : S_DEL_LR_MERGE]++;
+        ++R.n_lev;
+        R.n_nomove += c->b[10];
         const u32 ymax = R.BK(A)[K - 1];
         const u32 jx = x - base, jy = y - base;
         R.release(sl); R.release(sr);
         ns[jx] = B; mn[jx] = R.BK(B)[0]; mx[jx] = R.BK(B)[K - 1];
         ns[jy] = sy; pend[jy] = 1;
         if (ymax <= b.cmin) {  // l.12 swap: cur <- Y (pushed up), the carried keys sink on
-          c->st[S_DEL_CY_SWAP]++;
+          ++R.n_swap;
           R.push_up(A, up);
           push_old = A;
           R.send((u32)i, MK_B, 0, 0, b.src, b.cmin, b.cmax);
@@ -978,6 +997,7 @@ __device__ void ds_level(DsRole<K, V>& R, const u64 m) {
   // ---- end: pending pushes landed, write the owned nodes back
   if (tid == 0) {
     R.tacc(0, t_start);
+    R.flush_counts();
     asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
     for (u32 j = 0; j < cnt; ++j) {
       const u32 n = base + j;
@@ -1077,14 +1097,14 @@ __device__ void ds_stager(DsRole<K, V>& R, const u64 m) {
         R.release(A); R.release(B);
         st_rel_cta(&c->sq_ret, (u32)i + 1u);
       } else {
-        c->st[S_DEL_LEVELS]++;
-        c->st[c->b[10] ? S_DEL_LR_NOMOVE : S_DEL_LR_MERGE]++;
+        ++R.n_lev;
+        R.n_nomove += c->b[10];
         st_rel_cta(&c->sq_ret, (u32)i + 1u);  // the staged children were only split inputs
         // x <- X: HBM write-back, then UNLOCK(x) (helper B, l.11); it frees slot B
         sq_req<K, V>(R, &c->wq_head, &c->wq_done, c->wq, WQ_WB, x, B, R.BK(B)[0], R.BK(B)[K - 1]);
         const u32 ymax = R.BK(A)[K - 1];
         if (ymax <= b.cmin) {  // l.12 swap: cur <- Y, the carried keys go on to y's walker
-          c->st[S_DEL_CY_SWAP]++;
+          ++R.n_swap;
           R.push_up(A, up);
           push_old = A;
           if (b.src & DS_PULL) {  // on chip above: pull them and store them in y's HBM copy
@@ -1144,6 +1164,7 @@ __device__ void ds_stager(DsRole<K, V>& R, const u64 m) {
   }
   if (tid == 0) {
     R.tacc(0, t_start);
+    R.flush_counts();
     asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
   }
 }
