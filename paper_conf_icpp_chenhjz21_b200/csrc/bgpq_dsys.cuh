@@ -348,9 +348,11 @@ struct DsRole {
 };
 
 // All NT compute threads: SORT_SPLIT of two full K-batches, X = K smallest, Y = rest.
-template <int K, bool V>
+// LEAD = false where the caller's own CTA barrier directly precedes the call (only broadcast
+// words were read since): the leading barrier would be a second one back to back.
+template <int K, bool V, bool LEAD = true>
 __device__ __forceinline__ void ds_split(DsRole<K, V>& R, u32 z, u32 w, u32 x, u32 y) {
-  cta_bar<DS_NT>();
+  if (LEAD) cta_bar<DS_NT>();
   sort_split<K, DS_NT, V>(R.BK(z), R.BV(z), K, R.BK(w), R.BV(w), K, K, R.BK(x), R.BV(x), R.BK(y), R.BV(y));
   cta_bar<DS_NT>();
 }
@@ -469,7 +471,7 @@ __device__ void ds_r0(DsRole<K, V>& R, const u64 m) {
     if (c->b[0]) continue;
     const u32 s2 = c->b[1], s3 = c->b[2], A = c->b[3], B = c->b[4];
     const ull t3 = R.tnow();
-    ds_split<K, V>(R, s2, s3, A, B);  // l.10: (Heap[y], Heap[x]) <- SORT_SPLIT(l, r)
+    ds_split<K, V, false>(R, s2, s3, A, B);  // l.10: (Heap[y], Heap[x]) <- SORT_SPLIT(l, r)
     if (tid == 0) R.tacc(3, t3);
     if (tid == 0) {
       const u32 x = c->b[5], y = c->b[6], sy = c->b[7], t = c->b[8], rmin = c->b[9], rmax = c->b[10];
@@ -493,7 +495,7 @@ __device__ void ds_r0(DsRole<K, V>& R, const u64 m) {
     cta_bar<DS_NT>();
     if (c->b[15]) {  // rare: a real (cur, y) merge at the root
       const u32 r = c->b[11], lo = c->b[12], hi = c->b[13];
-      ds_split<K, V>(R, r, A, lo, hi);
+      ds_split<K, V, false>(R, r, A, lo, hi);
       if (tid == 0) {
         // C1 stays in slot hi; the level that needs its content pulls it (DS_PULL)
         R.pull_publish();
@@ -638,7 +640,7 @@ __device__ void ds_r0_mixed(DsRole<K, V>& R, const u64 m) {
     }
     cta_bar<DS_NT>();
     if (c->b[0] == 2) {
-      ds_split<K, V>(R, c->b[1], c->b[2], c->b[3], c->b[4]);
+      ds_split<K, V, false>(R, c->b[1], c->b[2], c->b[3], c->b[4]);
       if (tid == 0) {
         R.release(ns[1]); R.release(it);
         ns[1] = c->b[3]; it = c->b[4];
@@ -662,7 +664,7 @@ __device__ void ds_r0_mixed(DsRole<K, V>& R, const u64 m) {
     }
     cta_bar<DS_NT>();
     if (c->b[0] == 2) {
-      ds_split<K, V>(R, c->b[1], c->b[2], c->b[3], c->b[4]);
+      ds_split<K, V, false>(R, c->b[1], c->b[2], c->b[3], c->b[4]);
       if (tid == 0) {
         R.release(ns[d1]); R.release(it);
         ns[d1] = c->b[3]; it = c->b[4];
@@ -712,7 +714,7 @@ __device__ void ds_r0_mixed(DsRole<K, V>& R, const u64 m) {
     if (c->b[0]) continue;
     const u32 s2 = c->b[1], s3 = c->b[2], A = c->b[3], B = c->b[4];
     const ull t3 = R.tnow();
-    ds_split<K, V>(R, s2, s3, A, B);  // l.10
+    ds_split<K, V, false>(R, s2, s3, A, B);  // l.10
     if (tid == 0) R.tacc(3, t3);
     if (tid == 0) {
       const u32 x = c->b[5], y = c->b[6], sy = c->b[7];
@@ -740,7 +742,7 @@ __device__ void ds_r0_mixed(DsRole<K, V>& R, const u64 m) {
     cta_bar<DS_NT>();
     if (c->b[15]) {
       const u32 r = c->b[11], lo = c->b[12], hi = c->b[13];
-      ds_split<K, V>(R, r, A, lo, hi);
+      ds_split<K, V, false>(R, r, A, lo, hi);
       if (tid == 0) {
         R.pull_publish();  // C1 stays in slot hi until a lower level pulled it
         R.send((u32)i, MK_B, 0, 0, R.pull_ref(hi), R.BK(hi)[0], R.BK(hi)[K - 1]);
@@ -885,7 +887,7 @@ __device__ void ds_level(DsRole<K, V>& R, const u64 m) {
     if (c->b[0]) continue;
     const u32 sl = c->b[1], sr = c->b[2], A = c->b[3], B = c->b[4];
     const ull t3 = R.tnow();
-    ds_split<K, V>(R, sl, sr, A, B);  // l.10 (speculative until message b)
+    ds_split<K, V, false>(R, sl, sr, A, B);  // l.10 (speculative until message b)
     if (tid == 0) {
       R.segmark(4);
       R.tacc(3, t3);
@@ -1070,7 +1072,7 @@ __device__ void ds_stager(DsRole<K, V>& R, const u64 m) {
     if (c->b[0]) continue;
     const u32 sl = c->b[1], sr = c->b[2], A = c->b[3], B = c->b[4];
     const ull t3 = R.tnow();
-    ds_split<K, V>(R, sl, sr, A, B);
+    ds_split<K, V, false>(R, sl, sr, A, B);
     if (tid == 0) {
       R.tacc(3, t3);
       const u32 x = c->b[5], y = c->b[6], up = c->b[9], minc = c->b[13], l = c->b[11], r = c->b[12];
