@@ -152,6 +152,12 @@ __device__ __forceinline__ void bulk_s2cl(u32 dst, const void* src, u32 bytes, u
   asm volatile("cp.async.bulk.shared::cluster.shared::cta.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
                "r"(smem_addr(src)), "r"(bytes), "r"(bar) : "memory");
 }
+// 16-B asynchronous store into another CTA's shared memory that completes its bytes on that
+// CTA's mbarrier (st.async, sm_90+): the message transport of the cluster engine
+__device__ __forceinline__ void st_async_v4(u32 addr, u32 a, u32 b, u32 c, u32 d, u32 bar) {
+  asm volatile("st.async.shared::cluster.mbarrier::complete_tx::bytes.v4.b32 [%0], {%1, %2, %3, %4}, [%5];"
+               ::"r"(addr), "r"(a), "r"(b), "r"(c), "r"(d), "r"(bar) : "memory");
+}
 __device__ __forceinline__ void cluster_sync_all() {
   asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
 }
@@ -278,11 +284,11 @@ struct DsRole {
     while (out_seq - *reinterpret_cast<volatile u32*>(&c->consumed) >= DS_RING - DS_CREDIT) {}
     const u32 e = out_seq % DS_RING;
     const u32 dst = rank + 1;
-    DsMsg& m = c->stage[e];
-    m.op = op; m.kind = kind; m.y = y; m.slot = slot; m.src = src; m.cmin = cmin; m.cmax = cmax; m.pad = flags;
-    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-    bulk_s2cl(cl_map(&c->inbox[e], dst), &m, (u32)sizeof(DsMsg), cl_map(&c->inbar[e], dst));
-    asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+    // two 16-B remote async stores, each completing its bytes on the receiver's armed inbox
+    // barrier (no staging copy, no proxy fence, no bulk group)
+    const u32 ia = cl_map(&c->inbox[e], dst), ib = cl_map(&c->inbar[e], dst);
+    st_async_v4(ia, op, kind, y, slot, ib);
+    st_async_v4(ia + 16u, src, cmin, cmax, flags, ib);
     ++out_seq;
     tacc(5, t0);
   }
@@ -292,11 +298,9 @@ struct DsRole {
     while (out_seq2 - *reinterpret_cast<volatile u32*>(&c->aconsumed) >= DS_RING - DS_CREDIT) {}
     const u32 e = out_seq2 % DS_RING;
     const u32 dst = rank + 1;
-    DsMsg& m = c->astage[e];
-    m.op = op; m.kind = kind; m.y = y; m.slot = slot; m.src = 0; m.cmin = 0; m.cmax = 0; m.pad = 0;
-    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-    bulk_s2cl(cl_map(&c->ainbox[e], dst), &m, (u32)sizeof(DsMsg), cl_map(&c->ainbar[e], dst));
-    asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+    const u32 ia = cl_map(&c->ainbox[e], dst), ib = cl_map(&c->ainbar[e], dst);
+    st_async_v4(ia, op, kind, y, slot, ib);
+    st_async_v4(ia + 16u, 0u, 0u, 0u, 0u, ib);
     ++out_seq2;
     tacc(5, t0);
   }
