@@ -2,8 +2,8 @@
 # Evidence of the late round-2 build (under gpurun, one GPU): bench line, ncu launch lists of the
 # bench and of one C2 mixed call, ncu --set full captures of the DELETEMIN cluster kernel, the
 # INSERT pipeline kernel and the mixed call's cluster kernel; summaries + CSV exports.
-cd "$GRAFT_REPO_ROOT"; mkdir -p gpurun_out/late
-O=gpurun_out/late
+cd "$GRAFT_REPO_ROOT"; mkdir -p ${OUT:-gpurun_out/late}
+O=${OUT:-gpurun_out/late}
 NCU=/usr/local/cuda/bin/ncu
 timeout 900 python bench.py --steps 5 --warmup 3 > $O/bench.log 2>&1; echo "bench rc=$?"
 timeout 600 python tools/mix_once.py > $O/mix_once.log 2>&1 || { echo "mix_once failed"; exit 1; }
