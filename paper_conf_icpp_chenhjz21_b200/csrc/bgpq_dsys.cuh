@@ -35,8 +35,9 @@
 
 namespace bgpqd {
 
-constexpr int DS_NT = 512;             // compute threads per CTA
-constexpr int DS_BLOCK = DS_NT + 64;   // + 2 helper warps (roles) / lock warp + idle warp (walkers)
+constexpr int DS_NT = 512;             // split threads per role CTA (= walker compute threads)
+constexpr int DS_NC = DS_NT + 32;      // role CTAs: control warp 0 (thread 0 decides) + split warps 1-16
+constexpr int DS_BLOCK = DS_NC + 64;   // + 2 helper warps (roles) / lock warp + idle warps (walkers)
 constexpr int DS_CL = 5;               // cluster size: steps of depths 0 .. DS_CL-1 in the cluster
 constexpr int DS_NSLOT = 24;           // node slots per role CTA
 constexpr u32 DS_MAXOWN = 1u << (DS_CL - 1);  // nodes the deepest owning level holds (depth DS_CL-1)
@@ -219,7 +220,7 @@ struct DsRole {
   __device__ __forceinline__ void pull_copy(u32 ref, u32 dst) const {
     const u32 owner = (ref >> 8) & 0xFFu, src = ref & 0xFFu;
     const u32 rk = cl_map(BK(src), owner);
-    for (int q = threadIdx.x; q < K / 4; q += DS_NT) {
+    for (int q = threadIdx.x; q < K / 4; q += DS_NC) {
       uint4 v;
       asm volatile("ld.shared::cluster.v4.u32 {%0, %1, %2, %3}, [%4];"
                    : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(rk + 16u * q) : "memory");
@@ -227,7 +228,7 @@ struct DsRole {
     }
     if (V) {
       const u32 rv = cl_map(BV(src), owner);
-      for (int q = threadIdx.x; q < K / 4; q += DS_NT) {
+      for (int q = threadIdx.x; q < K / 4; q += DS_NC) {
         uint4 v;
         asm volatile("ld.shared::cluster.v4.u32 {%0, %1, %2, %3}, [%4];"
                      : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(rv + 16u * q) : "memory");
@@ -354,11 +355,21 @@ struct DsRole {
 // All NT compute threads: SORT_SPLIT of two full K-batches, X = K smallest, Y = rest.
 // LEAD = false where the caller's own CTA barrier directly precedes the call (only broadcast
 // words were read since): the leading barrier would be a second one back to back.
+// The split runs on warps 1-16 while thread 0 (warp 0) runs `during` — the role's bookkeeping
+// that the split does not need (its path message to the level below, slot arming, ...).
+template <int K, bool V, bool LEAD = true, typename F>
+__device__ __forceinline__ void ds_split_h(DsRole<K, V>& R, u32 z, u32 w, u32 x, u32 y, F&& during) {
+  if (LEAD) cta_bar<DS_NC>();
+  if (threadIdx.x >= 32)
+    sort_split_t<K, DS_NT, V>((int)threadIdx.x - 32, R.BK(z), R.BV(z), K, R.BK(w), R.BV(w), K, K, R.BK(x), R.BV(x),
+                              R.BK(y), R.BV(y));
+  else if (threadIdx.x == 0)
+    during();
+  cta_bar<DS_NC>();
+}
 template <int K, bool V, bool LEAD = true>
 __device__ __forceinline__ void ds_split(DsRole<K, V>& R, u32 z, u32 w, u32 x, u32 y) {
-  if (LEAD) cta_bar<DS_NT>();
-  sort_split<K, DS_NT, V>(R.BK(z), R.BV(z), K, R.BK(w), R.BV(w), K, K, R.BK(x), R.BV(x), R.BK(y), R.BV(y));
-  cta_bar<DS_NT>();
+  ds_split_h<K, V, LEAD>(R, z, w, x, y, [] {});
 }
 
 // Number of full-K ops the engine executes (identical in every role CTA): the call's full
@@ -414,7 +425,7 @@ __device__ void ds_r0(DsRole<K, V>& R, const u64 m) {
     mbar_wait(&c->lbar, R.lph);
     R.lph ^= 1u;
   }
-  cta_bar<DS_NT>();
+  cta_bar<DS_NC>();
   u32 out_old = DS_NONE;  // slot whose output store may still be reading it
   // op i's K output keys from slot s (TMA bulk store; the slot is freed once it was read)
   auto output = [&](u64 i, u32 s) {
@@ -471,7 +482,7 @@ __device__ void ds_r0(DsRole<K, V>& R, const u64 m) {
         R.n_nomove += (mx[2] <= mn[3] || mx[3] <= mn[2]) ? 1u : 0u;
       }
     }
-    cta_bar<DS_NT>();
+    cta_bar<DS_NC>();
     if (c->b[0]) continue;
     const u32 s2 = c->b[1], s3 = c->b[2], A = c->b[3], B = c->b[4];
     const ull t3 = R.tnow();
@@ -496,7 +507,7 @@ __device__ void ds_r0(DsRole<K, V>& R, const u64 m) {
       ns[x] = B; mn[x] = R.BK(B)[0]; mx[x] = R.BK(B)[K - 1];
       ns[y] = sy; pend[y] = 1;
     }
-    cta_bar<DS_NT>();
+    cta_bar<DS_NC>();
     if (c->b[15]) {  // rare: a real (cur, y) merge at the root
       const u32 r = c->b[11], lo = c->b[12], hi = c->b[13];
       ds_split<K, V, false>(R, r, A, lo, hi);
@@ -508,7 +519,7 @@ __device__ void ds_r0(DsRole<K, V>& R, const u64 m) {
         else { ns[1] = lo; mn[1] = R.BK(lo)[0]; mx[1] = R.BK(lo)[K - 1]; }
         R.release(r); R.release(A);
       }
-      cta_bar<DS_NT>();
+      cta_bar<DS_NC>();
     }
   }
   // ---- end: wait for the last pushes, write the on-chip nodes back, update the header
@@ -588,7 +599,7 @@ __device__ void ds_r0_mixed(DsRole<K, V>& R, const u64 m) {
     R.lph ^= 1u;
     asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(lin0) : "l"(H.hdr + H_LIN) : "memory");
   }
-  cta_bar<DS_NT>();
+  cta_bar<DS_NC>();
   u32 out_old = DS_NONE;
   auto output = [&](u64 j, u32 s) {  // op j's K output keys from slot s (TMA bulk store)
     asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
@@ -642,7 +653,7 @@ __device__ void ds_r0_mixed(DsRole<K, V>& R, const u64 m) {
       c->b[0] = ra;
       if (ra == 2) { c->b[1] = ns[1]; c->b[2] = it; c->b[3] = R.alloc(); c->b[4] = R.alloc(); }
     }
-    cta_bar<DS_NT>();
+    cta_bar<DS_NC>();
     if (c->b[0] == 2) {
       ds_split<K, V, false>(R, c->b[1], c->b[2], c->b[3], c->b[4]);
       if (tid == 0) {
@@ -666,7 +677,7 @@ __device__ void ds_r0_mixed(DsRole<K, V>& R, const u64 m) {
       c->b[0] = da;
       if (da == 2) { c->b[1] = ns[d1]; c->b[2] = it; c->b[3] = R.alloc(); c->b[4] = R.alloc(); }
     }
-    cta_bar<DS_NT>();
+    cta_bar<DS_NC>();
     if (c->b[0] == 2) {
       ds_split<K, V, false>(R, c->b[1], c->b[2], c->b[3], c->b[4]);
       if (tid == 0) {
@@ -714,7 +725,7 @@ __device__ void ds_r0_mixed(DsRole<K, V>& R, const u64 m) {
         R.n_nomove += (mx[2] <= mn[3] || mx[3] <= mn[2]) ? 1u : 0u;
       }
     }
-    cta_bar<DS_NT>();
+    cta_bar<DS_NC>();
     if (c->b[0]) continue;
     const u32 s2 = c->b[1], s3 = c->b[2], A = c->b[3], B = c->b[4];
     const ull t3 = R.tnow();
@@ -743,7 +754,7 @@ __device__ void ds_r0_mixed(DsRole<K, V>& R, const u64 m) {
       ns[x] = B; mn[x] = R.BK(B)[0]; mx[x] = R.BK(B)[K - 1];
       ns[y] = sy; pend[y] = 1;
     }
-    cta_bar<DS_NT>();
+    cta_bar<DS_NC>();
     if (c->b[15]) {
       const u32 r = c->b[11], lo = c->b[12], hi = c->b[13];
       ds_split<K, V, false>(R, r, A, lo, hi);
@@ -754,7 +765,7 @@ __device__ void ds_r0_mixed(DsRole<K, V>& R, const u64 m) {
         else { ns[1] = lo; mn[1] = R.BK(lo)[0]; mx[1] = R.BK(lo)[K - 1]; }
         R.release(r); R.release(A);
       }
-      cta_bar<DS_NT>();
+      cta_bar<DS_NC>();
     }
   }
   // ---- end: the on-chip nodes back to HBM; heapSize is unchanged by every pair
@@ -838,9 +849,9 @@ __device__ void ds_level(DsRole<K, V>& R, const u64 m) {
     mbar_wait(&c->lbar, R.lph);
     R.lph ^= 1u;
   }
-  cta_bar<DS_NT>();
+  cta_bar<DS_NC>();
   u32 push_old = DS_NONE;  // slot whose push may still be reading it
-  u32 a_src = 0, a_cmin = 0, a_cmax = 0, early = 0;  // thread 0: the path message's refill-key info
+  u32 a_src = 0, a_cmin = 0, a_cmax = 0, early = 0, a_flags = 0;  // thread 0: the path message's refill-key info
   const ull t_start = R.tnow();
   if (tid == 0) R.tseg = clock64();
   for (u64 i = 0; i < m; ++i) {
@@ -875,23 +886,27 @@ __device__ void ds_level(DsRole<K, V>& R, const u64 m) {
         // level above swapped; with R the walk does not stop here (l.4) iff a.cmax > minc
         a_src = a.src; a_cmin = a.cmin; a_cmax = a.cmax;
         early = !(R.C.debug & 1048576u) && (a.pad & MA_EARLY) && a.cmax > minc;  // debug 1048576: off
-        const u32 sy = R.alloc();  // y's new content arrives here from the level below
-        R.arm_slot(sy);
-        R.send_path((u32)i, MK_A, y, sy, a.src, a.cmin, a.cmax, early ? MA_EARLY : 0u);
         const u32 A = R.alloc(), B = R.alloc();
         c->b[1] = ns[jl]; c->b[2] = ns[jr]; c->b[3] = A; c->b[4] = B; c->b[5] = x; c->b[6] = y;
-        c->b[7] = sy; c->b[9] = a.slot;
+        c->b[9] = a.slot;
+        a_flags = early ? MA_EARLY : 0u;
         c->b[10] = (mx[jl] <= mn[jr] || mx[jr] <= mn[jl]) ? 1u : 0u;
         c->b[13] = minc;
         R.segmark(2);
       }
     }
-    cta_bar<DS_NT>();
+    cta_bar<DS_NC>();
     if (tid == 0) R.segmark(3);
     if (c->b[0]) continue;
     const u32 sl = c->b[1], sr = c->b[2], A = c->b[3], B = c->b[4];
     const ull t3 = R.tnow();
-    ds_split<K, V, false>(R, sl, sr, A, B);  // l.10 (speculative until message b)
+    ds_split_h<K, V, false>(R, sl, sr, A, B, [&] {  // l.10 (speculative until message b)
+      // during the split: y's slot for the level below's push, and the path message to it
+      const u32 sy = R.alloc();
+      R.arm_slot(sy);
+      R.send_path((u32)i, MK_A, c->b[6], sy, a_src, a_cmin, a_cmax, a_flags);
+      c->b[7] = sy;
+    });
     if (tid == 0) {
       R.segmark(4);
       R.tacc(3, t3);
@@ -973,12 +988,12 @@ __device__ void ds_level(DsRole<K, V>& R, const u64 m) {
       }
       }
     }
-    cta_bar<DS_NT>();
+    cta_bar<DS_NC>();
     if (tid == 0) R.segmark(9);
     if (c->b[14] == 2) {  // stop at cur with carried keys on chip above: pull, push up
       const u32 s2 = c->b[4], up = c->b[9], ref = c->b[15];
       R.pull_copy(ref, s2);
-      cta_bar<DS_NT>();
+      cta_bar<DS_NC>();
       if (tid == 0) {
         R.pull_free(ref);
         R.push_up(s2, up);
@@ -997,7 +1012,7 @@ __device__ void ds_level(DsRole<K, V>& R, const u64 m) {
         R.pull_publish();  // the new carried keys stay in slot hi until a lower level pulled them
         R.send((u32)i, MK_B, 0, 0, R.pull_ref(hi), R.BK(hi)[0], R.BK(hi)[K - 1]);
       }
-      cta_bar<DS_NT>();
+      cta_bar<DS_NC>();
     }
   }
   // ---- end: pending pushes landed, write the owned nodes back
@@ -1072,7 +1087,7 @@ __device__ void ds_stager(DsRole<K, V>& R, const u64 m) {
         c->b[11] = l; c->b[12] = r;
       }
     }
-    cta_bar<DS_NT>();
+    cta_bar<DS_NC>();
     if (c->b[0]) continue;
     const u32 sl = c->b[1], sr = c->b[2], A = c->b[3], B = c->b[4];
     const ull t3 = R.tnow();
@@ -1128,11 +1143,11 @@ __device__ void ds_stager(DsRole<K, V>& R, const u64 m) {
         }
       }
     }
-    cta_bar<DS_NT>();
+    cta_bar<DS_NC>();
     if (c->b[14] == 2 || c->b[14] == 3) {  // carried keys on chip above: pull them
       const u32 s2 = c->b[4], ref = c->b[15], mode = c->b[14];
       R.pull_copy(ref, s2);
-      cta_bar<DS_NT>();
+      cta_bar<DS_NC>();
       if (tid == 0) {
         R.pull_free(ref);
         if (mode == 2) {  // stop at cur: cur <- the carried keys
@@ -1146,7 +1161,7 @@ __device__ void ds_stager(DsRole<K, V>& R, const u64 m) {
           sq_req<K, V>(R, &c->wq_head, &c->wq_done, c->wq, WQ_COMMIT, y, y, 0, 0);
         }
       }
-      cta_bar<DS_NT>();
+      cta_bar<DS_NC>();
     } else if (c->b[14]) {  // a real (cur, y) merge
       const u32 cs = c->b[4], lo = c->b[5], hi = c->b[6], Y = c->b[12], ref = c->b[15];
       if (ref & DS_PULL) R.pull_copy(ref, cs);
@@ -1161,7 +1176,7 @@ __device__ void ds_stager(DsRole<K, V>& R, const u64 m) {
         R.release(cs); R.release(Y); R.release(hi);
         sq_req<K, V>(R, &c->wq_head, &c->wq_done, c->wq, WQ_COMMIT, y, y, 0, 0);
       }
-      cta_bar<DS_NT>();
+      cta_bar<DS_NC>();
     }
     if (tid == 0) {  // slots the write-back helper finished with
       const u32 fr = atomicExch(&c->wb_free, 0u);
@@ -1310,11 +1325,11 @@ __global__ void __cluster_dims__(DS_CL, 1, 1) __launch_bounds__(DS_BLOCK, 1)
     __syncthreads();
     cluster_sync_all();  // every barrier of the cluster initialised before any remote copy
     const bool stager = R.rank == DS_CL - 1;
-    if (threadIdx.x >= DS_NT) {
-      if (threadIdx.x == DS_NT) {
+    if (threadIdx.x >= DS_NC) {
+      if (threadIdx.x == DS_NC) {
         if (R.rank == 0) { if (C.mode != MODE_MIXED) ds_r0_helper<K, V>(R, m); }
         else if (stager) ds_stage_helper<K, V>(R, m);
-      } else if (threadIdx.x == DS_NT + 32 && stager) {
+      } else if (threadIdx.x == DS_NC + 32 && stager) {
         ds_wb_helper<K, V>(R);
       }
     } else {
@@ -1328,7 +1343,7 @@ __global__ void __cluster_dims__(DS_CL, 1, 1) __launch_bounds__(DS_BLOCK, 1)
       } else if (threadIdx.x == 0 && R.rank == 0) {
         *reinterpret_cast<volatile u64*>(D.op_base) = 0;
       }
-      cta_bar<DS_NT>();
+      cta_bar<DS_NC>();
       if (threadIdx.x == 0) st_rel_cta(&c->quit, 1u);
     }
     __syncthreads();

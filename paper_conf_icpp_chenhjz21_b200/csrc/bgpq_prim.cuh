@@ -774,6 +774,26 @@ __device__ __forceinline__ void sort_split(const u32* zk, const u32* zv, int na,
   cta_merge_win<K, NTM, V>(zk, zv, na, wk, wv, nb, ma, xk, xv, yk, yv);
 }
 
+// sort_split run by a group of NT threads whose index in the group is t (the group need not
+// start at thread 0; the bitonic path synchronises on named barrier BAR_BITONIC of NB threads)
+template <int K, int NT, bool V>
+__device__ __forceinline__ void sort_split_t(const int t, const u32* zk, const u32* zv, int na, const u32* wk,
+                                             const u32* wv, int nb, int ma, u32* xk, u32* xv, u32* yk, u32* yv) {
+#ifndef BGPQ_NO_BITONIC
+  if constexpr (!V) {
+    constexpr int NB = (K < 512 ? K : 512) <= NT ? (K < 512 ? K : 512) : 0;
+    if constexpr (NB >= 64 && K >= BITONIC_MIN_K) {
+      if (na == K && nb == K && ma == K) {
+        if (t < NB) bitonic_split_full<K, NB, false>(t, BAR_BITONIC, zk, zv, wk, wv, xk, xv, yk, yv);
+        return;
+      }
+    }
+  }
+#endif
+  constexpr int NTM = (2 * K / 4 <= NT) ? 2 * K / 4 : NT;
+  grp_merge_win<K, NTM, V>(t, zk, zv, na, wk, wv, nb, ma, xk, xv, yk, yv);
+}
+
 // One pass of a bottom-up merge sort: merge sorted runs [2q*run, (2q+1)*run) and
 // [(2q+1)*run, (2q+2)*run) of src (n entries, n a multiple of 2*run) into dst, by co-ranking.
 template <int KMAX, int NT, bool V>
