@@ -93,7 +93,10 @@ class _Search:
 class KnapsackSearch(_Search):
     """0-1 knapsack branch and bound (R23) on the current GPU."""
     maximize = True
-    DEFAULT_CTAS = 64  # C4: 1.50 s at 64 CTAs vs 1.79 s with all 148
+    # C4: 1.58-1.64 s in 6 of 6 solves at 16 CTAs; at 32 / 64 CTAs the relaxed best-first order
+    # expands up to 10x more nodes in some solves (1.4-13 s / 1.8-16 s; one 64-CTA solve ran
+    # > 2 min), a heavy tail from late incumbents (tools/ab_ks.py, one B200)
+    DEFAULT_CTAS = 16
 
     def __init__(self, w: np.ndarray, p: np.ndarray, C: int, K: int = 1024, capacity: int = 1 << 27,
                  ctas: int | None = None):
