@@ -678,19 +678,10 @@ __device__ void ds_r0_mixed(DsRole<K, V>& R, const u64 m) {
       if (da == 2) { c->b[1] = ns[d1]; c->b[2] = it; c->b[3] = R.alloc(); c->b[4] = R.alloc(); }
     }
     cta_bar<DS_NC>();
-    if (c->b[0] == 2) {
-      ds_split<K, V, false>(R, c->b[1], c->b[2], c->b[3], c->b[4]);
-      if (tid == 0) {
-        R.release(ns[d1]); R.release(it);
-        ns[d1] = c->b[3]; it = c->b[4];
-        mn[d1] = R.BK(ns[d1])[0]; mx[d1] = R.BK(ns[d1])[K - 1];
-        imin = R.BK(it)[0]; imax = R.BK(it)[K - 1];
-      }
-    }
-    // ---- DELETEMIN: the root's keys are its output (Alg.2 l.22), the refill keys are the
-    // INSERT's items (the MARKED hand-off, l.7-12), then Alg.3 at the root as in ds_r0
-    if (tid == 0) {
-      const u32 o1 = 5u - d1;  // the other depth-1 node, read by the depth-0 step only
+    // thread 0's work for the DELETEMIN that the INSERT's depth-1 split does not need: the other
+    // depth-1 node's push (op i-1's y1) and the op tickets — overlapped with that split
+    const u32 o1 = 5u - d1;
+    auto pre_del = [&] {
       if (pend[o1]) {
         const ull t2 = R.tnow();
         R.wait_pushed(ns[o1]);
@@ -699,12 +690,27 @@ __device__ void ds_r0_mixed(DsRole<K, V>& R, const u64 m) {
         mx[o1] = R.BK(ns[o1])[K - 1];
         R.tacc(2, t2);
       }
-
       if (C.lin_ticket) {
         st_relaxed_u64(reinterpret_cast<u64*>(C.lin_ticket) + 2 * i, lin0 + 2 * i);
         st_relaxed_u64(reinterpret_cast<u64*>(C.lin_ticket) + jd, lin0 + jd);
       }
       st_relaxed(C.op_count + jd, (u32)K);
+    };
+    if (c->b[0] == 2) {
+      ds_split_h<K, V, false>(R, c->b[1], c->b[2], c->b[3], c->b[4], pre_del);
+      if (tid == 0) {
+        R.release(ns[d1]); R.release(it);
+        ns[d1] = c->b[3]; it = c->b[4];
+        mn[d1] = R.BK(ns[d1])[0]; mx[d1] = R.BK(ns[d1])[K - 1];
+        imin = R.BK(it)[0]; imax = R.BK(it)[K - 1];
+      }
+    } else if (tid == 0) {
+      pre_del();
+    }
+    // ---- DELETEMIN: the root's keys are its output (Alg.2 l.22), the refill keys are the
+    // INSERT's items (the MARKED hand-off, l.7-12), then Alg.3 at the root as in ds_r0
+    if (tid == 0) {
+
       if (!rz) output(jd, ns[1]);
       const u32 minc = mn[2] < mn[3] ? mn[2] : mn[3];
       if (imax <= minc) {  // l.4: stop at the root — root <- the refill keys
