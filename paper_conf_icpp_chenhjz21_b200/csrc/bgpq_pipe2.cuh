@@ -28,7 +28,7 @@ namespace bgpqd {
 
 constexpr u32 P2_PIN = 4;     // in-ring entries (H1 -> compute)
 constexpr u32 P2_RQ = 16;     // H2 request ring
-constexpr u32 P2_H2D = 4;     // H2 requests in flight (bulk groups)
+constexpr u32 P2_H2D = 8;     // H2 requests in flight (bulk groups), retired as one batch
 // smem node slots per stage: 24, fewer for the largest nodes (the stage needs >= 12: root,
 // pBuffer, the in-ring entries' item and node slots, the sends in flight)
 template <int K, bool V>
@@ -248,6 +248,13 @@ struct Pipe2 {
     auto retire = [&](u32 keep) {  // more than `keep` requests in flight: complete all of them
       if (inflight <= keep) return;
       const ull t0 = tm ? clock64() : 0ull;
+      // the source slots come back as soon as the copies have read them (a node write-back's
+      // HBM write takes far longer to complete than its shared-memory read)
+      asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+      for (u32 q = 0; q < inflight; ++q) {
+        u32* f = pc->fq[(head_i + q) % D];
+        if (f[4] != P2_NONE) { release(f[4]); f[4] = P2_NONE; }
+      }
       asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
       const ull t1 = tm ? clock64() : 0ull;
       if (tm) w_wg += t1 - t0;
@@ -258,7 +265,6 @@ struct Pipe2 {
       while (inflight) {
         const u32* f = pc->fq[head_i % D];
         const u32 type = f[0], a = f[1], b = f[2], c = f[3];
-        if (f[4] != P2_NONE) release(f[4]);  // the smem source was read
         if (type == P2_WB) {
           st_relaxed(&H.meta[a].kmin, f[5]);
           st_relaxed(&H.meta[a].kmax, f[6]);
