@@ -1,7 +1,7 @@
 #!/bin/bash
 # Late round-2 evidence (under gpurun): C3 x K sweep, utilisation sweep (mix at three prefills),
 # application benches, w = 8 bench
-cd "$GRAFT_REPO_ROOT"; O=gpurun_out/late2; mkdir -p $O
+cd "$GRAFT_REPO_ROOT"; O=${OUT:-gpurun_out/late2}; mkdir -p $O
 : > $O/sweep_c3.jsonl
 for d in uniform ascending descending gaussian; do
   for k in 128 256 512 1024 2048 4096; do
